@@ -1,0 +1,156 @@
+/*
+ * tfhe_b200.h -- C ABI of the B200-native TFHE gate-bootstrapping library (libtfhe_b200.so).
+ *
+ * What it does: the data-parallel hot path of PyTFHE's execution backend (Ma, Xu, Wills, ISPASS 2023) --
+ * batched bootstrapped gates over the independent gates of one level of a levelised netlist.
+ *   P:N = /root/reference/PAPER.md line N.  "Cn" / "Rn" = readings listed in DESIGN.md.
+ *   - Problem statement: the backend exposes "bootstrapped gate computations (e.g., bootstrapped-NAND,
+ *     bootstrapped-XOR)" on ciphertexts; the key is broadcast to the workers before traversal
+ *     (P:239); a program is a DAG of gates traversed level by level by Algorithm 1 and the
+ *     output nodes are returned.
+ *   - A bootstrapped gate = linear combination -> blind rotation -> sample extraction ->
+ *     key switching, at the TFHE default 128-bit parameters: n=630 N=1024 k=1 l=3 Bgbit=7,
+ *     KS t=8 base 4.  Only this parameter set is compiled; anything else -> TB_EUNSUPPORTED.
+ *
+ * Data types.  Torus32 values are uint32_t.  An LWE ciphertext is a[0..629], b (631 words) stored in a row
+ * of `stride` >= 631 words.  Keys are produced by the client (secret keys never reach this library).
+ *
+ * Conventions.
+ *   - Every function returns int status: 0 = TB_OK, < 0 = error; nothing throws across the ABI.  On error
+ *     tb_last_error() returns a thread-local message.
+ *   - Pointers named dev_* / wires / out / ca / cb / cc are DEVICE pointers (cudaMalloc or torch tensors'
+ *     data_ptr()) on the context's device; host_* pointers are host memory (pinned for async copies).
+ *   - The caller owns every ciphertext buffer; the context owns keys and scratch.
+ *   - Run calls (tb_gates, tb_run_level, tb_run_netlist) are stream-ordered on `stream` and never
+ *     synchronise the device.  Load calls and tb_gates_host synchronise.
+ *   - Thread-compatible: a context may be used by one host thread / one stream at a time (it owns
+ *     scratch buffers that a second concurrent stream would race on).
+ */
+#ifndef TFHE_B200_H
+#define TFHE_B200_H
+#include <stddef.h>
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* tb_stream;   /* == cudaStream_t; NULL = legacy default stream */
+
+typedef struct {
+    int32_t n, N, k, l, Bgbit, ks_t, ks_basebit;
+} tb_params;
+
+typedef struct tb_ctx tb_ctx;
+
+enum {
+    TB_OK = 0,
+    TB_EINVAL = -1,        /* null pointer, bad count / stride / index / gate code */
+    TB_EUNSUPPORTED = -2,  /* parameter set other than the compiled one, or device is not sm_100 */
+    TB_ENOKEYS = -3,       /* a run call before tb_load_bk and tb_load_ksk */
+    TB_ECUDA = -4,         /* CUDA runtime error (message in tb_last_error) */
+    TB_ENOMEM = -5         /* device or host allocation failed */
+};
+
+/* Gate codes = the 4-bit PyTFHE type field, read as the truth table f(a,b) at bit (2a+b) (Fig. 5;
+ * reading C15; XOR = 0110 is the one code the paper prints).  MUX is a 3-input extension. */
+enum tb_gate {
+    TB_NOR = 1, TB_ANDNY = 2, TB_NOT = 3, TB_ANDYN = 4, TB_XOR = 6, TB_NAND = 7, TB_AND = 8,
+    TB_XNOR = 9, TB_ORNY = 11, TB_ORYN = 13, TB_OR = 14, TB_MUX = 16
+};
+
+/* Default parameters (n=630, N=1024, k=1, l=3, Bgbit=7, ks_t=8, ks_basebit=2). */
+tb_params tb_default_params(void);
+
+/* Create a context on CUDA device `cuda_device`.  Fails with TB_EUNSUPPORTED for any other parameter set
+ * or a device without compute capability 10.0.  *out receives the context. */
+int tb_ctx_create(const tb_params* params, int cuda_device, tb_ctx** out);
+int tb_ctx_destroy(tb_ctx* ctx);
+
+/* Bootstrapping key, HOST pointer, torus layout [i < n][row r = bloc*l + j < 2l][poly < 2][N] u32
+ * (n_words must equal n*2l*2*N = 7,741,440).  The library splits each coefficient into 3 signed parts,
+ * transforms them to the NTT domain on the device (92.9 MB resident) and keeps no host copy.  Synchronous. */
+int tb_load_bk(tb_ctx* ctx, const uint32_t* host_bk, size_t n_words);
+/* Key-switching key, HOST pointer, layout [i < N][j < t][d < 4][n+1] u32 (n_words = 10,338,304).  Digit-0
+ * rows (encryptions of 0, never read, C9) are dropped and rows padded to 632 words (62.1 MB).  Synchronous. */
+int tb_load_ksk(tb_ctx* ctx, const uint32_t* host_ksk, size_t n_words);
+
+/* Batched single-type bootstrapped gates over DEVICE arrays: out[g] = gate(ca[g], cb[g] [, cc[g]]) for
+ * g < count, rows `stride` words apart in every array.  cb is ignored for TB_NOT; cc is used by TB_MUX
+ * only.  out must not alias the inputs.  Async on `stream`. */
+int tb_gates(tb_ctx* ctx, int gate, const uint32_t* ca, const uint32_t* cb, const uint32_t* cc,
+             uint32_t* out, int64_t count, int64_t stride, tb_stream stream);
+
+/* Same, HOST arrays (end-to-end path: host->device copies, gates, device->host copy, synchronise).  Uses
+ * context-owned device staging buffers. */
+int tb_gates_host(tb_ctx* ctx, int gate, const uint32_t* host_ca, const uint32_t* host_cb,
+                  const uint32_t* host_cc, uint32_t* host_out, int64_t count, int64_t stride);
+
+/* ---- netlists (Algorithm 1) ------------------------------------------------------------
+ * Wire ids: [0, n_inputs) are the program inputs, n_inputs + g is the output of gate g.  type[g] is a gate
+ * code; in1 = -1 for NOT, in2 = -1 unless MUX.  Gates may be listed in any order (no topological order is
+ * assumed, C15); a cycle or an out-of-range wire -> TB_EINVAL. */
+typedef struct {
+    int64_t n_inputs;
+    int64_t n_gates;
+    const int32_t* type;
+    const int64_t* in0;
+    const int64_t* in1;
+    const int64_t* in2;
+} tb_netlist;
+
+/* Algorithm 1 on the host: level_of_gate[g] = 1 + max(level of its inputs), inputs at level 0 -- the
+ * iteration of the while loop in which g first enters C - finished.  Writes *n_levels. */
+int tb_levelise(const tb_netlist* net, int64_t* level_of_gate, int64_t* n_levels);
+
+typedef struct tb_dev_netlist tb_dev_netlist;   /* library-owned device copy of a levelised netlist */
+
+/* Levelise, renumber wires so that every level's outputs form one contiguous block of rows (inputs first,
+ * then level 1, level 2, ...; within a level, gates in ascending original index), build the per-level
+ * lane and gate descriptors and upload them.  *out receives the handle. */
+int tb_netlist_upload(tb_ctx* ctx, const tb_netlist* net, tb_dev_netlist** out);
+int tb_netlist_free(tb_ctx* ctx, tb_dev_netlist* dnet);
+/* n_levels; n_rows = n_inputs + n_gates = rows a wire array must hold. */
+int tb_netlist_info(const tb_dev_netlist* dnet, int64_t* n_levels, int64_t* n_rows);
+/* row_of_wire[w] for every wire id w < n_inputs + n_gates (inputs map to themselves). */
+int tb_netlist_wire_rows(const tb_dev_netlist* dnet, int64_t* row_of_wire);
+/* first output row and number of gates (rows) of level `level` (1-based, 1..n_levels); also the number
+ * of bootstrapped gates and of blind-rotation lanes (MUX = 2 lanes, NOT = 0) in it. */
+int tb_netlist_level(const tb_dev_netlist* dnet, int64_t level, int64_t* row0, int64_t* n_gates,
+                     int64_t* n_boot, int64_t* n_lanes);
+/* Evaluate gates [g0, g1) of level `level` (indices within the level): reads input rows of `wires`,
+ * writes rows row0+g0 .. row0+g1-1.  `wires` is a DEVICE array of n_rows rows of `stride` words.  Async. */
+int tb_run_level(tb_ctx* ctx, const tb_dev_netlist* dnet, int64_t level, int64_t g0, int64_t g1,
+                 uint32_t* wires, int64_t stride, tb_stream stream);
+/* All levels in order on one device (single-GPU path).  Async. */
+int tb_run_netlist(tb_ctx* ctx, const tb_dev_netlist* dnet, uint32_t* wires, int64_t stride, tb_stream stream);
+
+/* ---- diagnostics used by the parity tests ---------------------------------------------------------- */
+/* Blind rotation + extraction only: out[g] (N+1 words, rows `out_stride` apart) = Extract(BlindRotate(
+ * ModSwitch(in[g]))) with test vector mu = 1/8 -- SURVEY 8(a) a2-a5 without the key switch.  Async. */
+int tb_bootstrap_wo_ks(tb_ctx* ctx, const uint32_t* in, int64_t in_stride, uint32_t* out, int64_t out_stride,
+                       int64_t count, tb_stream stream);
+/* Key switch only: out[g] (n+1 words) = KS(in[g]) for extracted samples in[g] (N+1 words).  Async. */
+int tb_keyswitch(tb_ctx* ctx, const uint32_t* in, int64_t in_stride, uint32_t* out, int64_t out_stride,
+                 int64_t count, tb_stream stream);
+/* Exact negacyclic product through the kernels' NTT (diagnostic): res[c] = sum over the 6 "rows" r of
+ * (digits[r] (x) polys[r])[c] mod 2^32, digits in [-64, 63], polys u32 torus.  All DEVICE pointers:
+ * digits [6][N] int32, polys [6][N] u32, res [N] u32.  Synchronous. */
+int tb_ntt_muladd6(tb_ctx* ctx, const int32_t* digits, const uint32_t* polys, uint32_t* res);
+
+/* Blind-rotation lanes per CTA (1..4, default 2); tuning knob, returns TB_EINVAL if out of range. */
+int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
+/* Device bytes a context holds for keys (BK NTT + KSK). */
+int tb_key_bytes(const tb_ctx* ctx, size_t* bytes);
+
+/* Integer-pipe microbenchmark (roofline denominator): runs the kernels' own lazy
+ * butterfly, register resident, on all SMs for `iters` iterations; returns butterflies/s and the 64-bit
+ * multiply-accumulate rate (MAC/s) measured with CUDA events.  Synchronous. */
+int tb_microbench(tb_ctx* ctx, int iters, double* butterflies_per_s, double* macs_per_s);
+
+const char* tb_last_error(void);
+const char* tb_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,230 @@
+"""paper_conf_ispass_maxw23_b200 -- B200-native batched TFHE gate bootstrapping (PyTFHE's hot path).
+
+Thin Python binding over the C ABI of libtfhe_b200.so (include/tfhe_b200.h); same names, argument
+marshalling only.  PyTorch provides device memory (ciphertexts live in int32 CUDA tensors whose bits are the
+u32 torus words), streams and process groups; every step of a gate runs in the sm_100a kernels.
+
+    ctx = Context()                      # cuda:0, tfhe-lib 128-bit parameters
+    ctx.load_keys(bk, ksk)               # host u32 arrays from the client's KeyGen
+    out = ctx.gates(NAND, ca, cb)        # batched bootstrapped gates
+    dnet = ctx.upload(netlist)           # Algorithm-1 levelisation + descriptors
+    ctx.run_netlist(dnet, wires)         # level by level on one GPU, or sharded over a process group
+
+P:N = /root/reference/PAPER.md line N.
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+import torch
+
+from . import _native, parallel
+from ._native import TBError, build
+from .netlist import (AND, ANDNY, ANDYN, BINARY_GATES, GATE_CODES, MUX, NAND, NOR, NOT, OR, ORNY, ORYN, XNOR, XOR,
+                      Netlist, read_pytfhe_binary, write_pytfhe_binary)
+
+N_LWE = 630            # n
+N_RING = 1024          # N
+CT_WORDS = N_LWE + 1   # 631 words per LWE ciphertext (2524 B = the paper's 2.46 KB)
+EXT_WORDS = N_RING + 1
+WIRE_STRIDE = 632      # default row stride of wire arrays (16-byte aligned rows)
+BK_WORDS = N_LWE * 6 * 2 * N_RING
+KSK_WORDS = N_RING * 8 * 4 * CT_WORDS
+
+__all__ = ["Context", "DevNetlist", "Netlist", "TBError", "build", "read_pytfhe_binary", "write_pytfhe_binary",
+           "GATE_CODES", "NAND", "AND", "OR", "NOR", "XOR", "XNOR", "ANDNY", "ANDYN", "ORNY", "ORYN", "NOT", "MUX",
+           "CT_WORDS", "WIRE_STRIDE", "BK_WORDS", "KSK_WORDS", "version"]
+
+
+def version() -> str:
+    return _native.lib().tb_version().decode()
+
+
+def _ptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _stream_handle(stream=None):
+    s = torch.cuda.current_stream() if stream is None else stream
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _check_dev(t: torch.Tensor, device: torch.device, name: str):
+    if t.device != device or t.dtype != torch.int32 or t.dim() != 2 or t.stride(1) != 1:
+        raise ValueError("%s must be a 2-D int32 tensor on %s with unit inner stride" % (name, device))
+
+
+class DevNetlist:
+    """Library-owned device copy of a levelised netlist (tb_netlist_upload)."""
+
+    def __init__(self, ctx: "Context", net: Netlist):
+        self.ctx, self.net = ctx, net
+        h = ctypes.c_void_p()
+        s = net.c_struct()
+        _native.check(_native.lib().tb_netlist_upload(ctx._h, ctypes.byref(s), ctypes.byref(h)))
+        self._h = h
+        nl, nr = ctypes.c_int64(), ctypes.c_int64()
+        _native.check(_native.lib().tb_netlist_info(h, ctypes.byref(nl), ctypes.byref(nr)))
+        self.n_levels, self.n_rows = int(nl.value), int(nr.value)
+        self.row_of_wire = np.zeros(net.n_wires, np.int64)
+        _native.check(_native.lib().tb_netlist_wire_rows(h, self.row_of_wire.ctypes.data))
+        self.levels = []          # (row0, n_gates, n_boot, n_lanes) per level 1..n_levels
+        for L in range(1, self.n_levels + 1):
+            v = [ctypes.c_int64() for _ in range(4)]
+            _native.check(_native.lib().tb_netlist_level(h, L, *[ctypes.byref(x) for x in v]))
+            self.levels.append(tuple(int(x.value) for x in v))
+
+    @property
+    def n_boot(self) -> int:
+        return sum(lv[2] for lv in self.levels)
+
+    def free(self):
+        if self._h:
+            _native.lib().tb_netlist_free(self.ctx._h, self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+class Context:
+    """One device, keys resident in HBM (BK in the NTT domain 92.9 MB, KSK 62.1 MB)."""
+
+    def __init__(self, device=0):
+        self.device = torch.device("cuda", device if isinstance(device, int) else torch.device(device).index or 0)
+        L = _native.lib()
+        p = L.tb_default_params()
+        h = ctypes.c_void_p()
+        _native.check(L.tb_ctx_create(ctypes.byref(p), self.device.index, ctypes.byref(h)))
+        self._h = h
+
+    # ---- keys (the public key is broadcast to the workers before traversal) ----
+    def load_bk(self, bk: np.ndarray):
+        bk = np.ascontiguousarray(bk, np.uint32).reshape(-1)
+        _native.check(_native.lib().tb_load_bk(self._h, bk.ctypes.data, bk.size))
+
+    def load_ksk(self, ksk: np.ndarray):
+        ksk = np.ascontiguousarray(ksk, np.uint32).reshape(-1)
+        _native.check(_native.lib().tb_load_ksk(self._h, ksk.ctypes.data, ksk.size))
+
+    def load_keys(self, bk: np.ndarray, ksk: np.ndarray):
+        self.load_bk(bk)
+        self.load_ksk(ksk)
+
+    def set_lanes_per_cta(self, lanes: int):
+        _native.check(_native.lib().tb_set_lanes_per_cta(self._h, lanes))
+
+    # ---- tensors ----
+    def empty(self, rows: int, stride: int = WIRE_STRIDE) -> torch.Tensor:
+        return torch.empty((rows, stride), dtype=torch.int32, device=self.device)
+
+    def to_device(self, cts: np.ndarray, stride: int = WIRE_STRIDE) -> torch.Tensor:
+        cts = np.asarray(cts, np.uint32)
+        t = torch.zeros((cts.shape[0], stride), dtype=torch.int32)
+        t[:, :cts.shape[1]] = torch.from_numpy(cts.view(np.int32))
+        return t.to(self.device)
+
+    @staticmethod
+    def to_host(t: torch.Tensor, words: int = CT_WORDS) -> np.ndarray:
+        return t[:, :words].cpu().numpy().view(np.uint32).copy()
+
+    # ---- batched gates (P:54 bootstrapped-Gate) ----
+    def gates(self, gate: int, ca: torch.Tensor, cb: torch.Tensor = None, cc: torch.Tensor = None,
+              out: torch.Tensor = None, stream=None) -> torch.Tensor:
+        _check_dev(ca, self.device, "ca")
+        for name, t in (("cb", cb), ("cc", cc)):
+            if t is not None:
+                _check_dev(t, self.device, name)
+                if t.shape != ca.shape or t.stride() != ca.stride():
+                    raise ValueError("%s must match ca's shape and stride" % name)
+        out = torch.empty_like(ca) if out is None else out
+        _check_dev(out, self.device, "out")
+        _native.check(_native.lib().tb_gates(self._h, gate, _ptr(ca), _ptr(cb), _ptr(cc), _ptr(out), ca.shape[0],
+                                             ca.stride(0), _stream_handle(stream)))
+        return out
+
+    def gates_host(self, gate: int, ca: np.ndarray, cb: np.ndarray = None, cc: np.ndarray = None) -> np.ndarray:
+        """End-to-end through host buffers (H2D, gates, D2H inside the call)."""
+        ca = np.ascontiguousarray(ca, np.uint32)
+        cb = None if cb is None else np.ascontiguousarray(cb, np.uint32)
+        cc = None if cc is None else np.ascontiguousarray(cc, np.uint32)
+        out = np.empty_like(ca)
+        vp = lambda a: None if a is None else a.ctypes.data
+        _native.check(_native.lib().tb_gates_host(self._h, gate, vp(ca), vp(cb), vp(cc), out.ctypes.data,
+                                                  ca.shape[0], ca.shape[1]))
+        return out
+
+    def bootstrap_wo_ks(self, cts: torch.Tensor, out: torch.Tensor = None, stream=None) -> torch.Tensor:
+        _check_dev(cts, self.device, "cts")
+        out = torch.empty((cts.shape[0], 1028), dtype=torch.int32, device=self.device) if out is None else out
+        _native.check(_native.lib().tb_bootstrap_wo_ks(self._h, _ptr(cts), cts.stride(0), _ptr(out), out.stride(0),
+                                                       cts.shape[0], _stream_handle(stream)))
+        return out
+
+    def keyswitch(self, ext: torch.Tensor, out: torch.Tensor = None, stream=None) -> torch.Tensor:
+        _check_dev(ext, self.device, "ext")
+        out = self.empty(ext.shape[0]) if out is None else out
+        _native.check(_native.lib().tb_keyswitch(self._h, _ptr(ext), ext.stride(0), _ptr(out), out.stride(0),
+                                                 ext.shape[0], _stream_handle(stream)))
+        return out
+
+    def ntt_muladd6(self, digits: torch.Tensor, polys: torch.Tensor) -> torch.Tensor:
+        res = torch.empty(N_RING, dtype=torch.int32, device=self.device)
+        _native.check(_native.lib().tb_ntt_muladd6(self._h, _ptr(digits.contiguous()), _ptr(polys.contiguous()),
+                                                   _ptr(res)))
+        return res
+
+    def microbench(self, iters: int = 4096):
+        b, m = ctypes.c_double(), ctypes.c_double()
+        _native.check(_native.lib().tb_microbench(self._h, iters, ctypes.byref(b), ctypes.byref(m)))
+        return b.value, m.value
+
+    def key_bytes(self) -> int:
+        v = ctypes.c_size_t()
+        _native.check(_native.lib().tb_key_bytes(self._h, ctypes.byref(v)))
+        return int(v.value)
+
+    # ---- netlists (Algorithm 1) ----
+    def upload(self, net: Netlist) -> DevNetlist:
+        return DevNetlist(self, net)
+
+    def wire_array(self, dnet: DevNetlist, slack_rows: int = 0, stride: int = WIRE_STRIDE) -> torch.Tensor:
+        return torch.zeros((dnet.n_rows + slack_rows, stride), dtype=torch.int32, device=self.device)
+
+    def run_level(self, dnet: DevNetlist, level: int, g0: int, g1: int, wires: torch.Tensor, stream=None):
+        _check_dev(wires, self.device, "wires")
+        _native.check(_native.lib().tb_run_level(self._h, dnet._h, level, g0, g1, _ptr(wires), wires.stride(0),
+                                                 _stream_handle(stream)))
+
+    def run_netlist(self, dnet: DevNetlist, wires: torch.Tensor, group=None, stream=None):
+        """Evaluate every level.  Without a process group: one device (tb_run_netlist).  With one: each
+        level's gates are split into R contiguous chunks, rank r evaluates chunk r, and the output rows are
+        all-gathered in place over NCCL before the next level."""
+        if group is None:
+            _check_dev(wires, self.device, "wires")
+            _native.check(_native.lib().tb_run_netlist(self._h, dnet._h, _ptr(wires), wires.stride(0),
+                                                       _stream_handle(stream)))
+            return
+        _check_dev(wires, self.device, "wires")
+        parallel.level_loop([(row0, ng) for row0, ng, _, _ in dnet.levels], wires,
+                            lambda L, g0, g1: self.run_level(dnet, L, g0, g1, wires, stream), group)
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _native.lib().tb_ctx_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def slack_rows(dnet: DevNetlist, world: int) -> int:
+    """Extra wire rows needed so every level's padded all-gather stays inside the array."""
+    return parallel.slack_rows([(row0, ng) for row0, ng, _, _ in dnet.levels], dnet.n_rows, world)

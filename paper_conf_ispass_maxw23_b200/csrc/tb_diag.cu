@@ -1,0 +1,178 @@
+// tb_diag.cu -- constant upload, the NTT-product diagnostic used by the unit parity test, and the
+// integer-pipe microbenchmark that gives the "alu" roofline denominator.
+#include "tb_kernels.cuh"
+#include "tb_ntt.cuh"
+
+namespace tb {
+
+int set_ntt_constants(const uint32_t* fw, const uint32_t* fwp, const uint32_t* iw, const uint32_t* iwp,
+                      const uint32_t* misc) {
+    if (cudaMemcpyToSymbol(c_fw, fw, 32 * 4) != cudaSuccess) return -1;
+    if (cudaMemcpyToSymbol(c_fwp, fwp, 32 * 4) != cudaSuccess) return -1;
+    if (cudaMemcpyToSymbol(c_iw, iw, 32 * 4) != cudaSuccess) return -1;
+    if (cudaMemcpyToSymbol(c_iwp, iwp, 32 * 4) != cudaSuccess) return -1;
+    if (cudaMemcpyToSymbol(c_misc, misc, 4 * 4) != cudaSuccess) return -1;
+    return 0;
+}
+
+// res = sum_{r<6} digits[r] (x) polys[r] mod 2^32 through the same field, split, transforms, MAC reduction
+// and lift that the blind-rotation kernel uses (one CTA, 6 warps).
+struct DiagSmem {
+    uint2 twF[31 * 32];
+    uint2 twI[31 * 32];
+    uint32_t d[kRows][kSlotWords];
+    uint32_t b[kRows][kParts][kSlotWords];
+    uint32_t o[kParts][kSlotWords];
+};
+
+__global__ void __launch_bounds__(192) ntt_muladd6_kernel(const int32_t* digits, const uint32_t* polys,
+                                                          uint32_t* res, const uint2* twF, const uint2* twI,
+                                                          uint32_t ninv, uint32_t ninvp) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    DiagSmem& S = *reinterpret_cast<DiagSmem*>(smem_raw);
+    const int lane = threadIdx.x & 31, r = threadIdx.x >> 5;
+    for (int k = threadIdx.x; k < 31 * 32; k += blockDim.x) {
+        S.twF[k] = twF[k];
+        S.twI[k] = twI[k];
+    }
+    __syncthreads();
+    uint32_t x[32];
+#pragma unroll
+    for (int j = 0; j < 32; j++) {
+        const int32_t dv = digits[r * kN + lane + 32 * j];
+        x[j] = dv < 0 ? (uint32_t)(dv + (int32_t)kP) : (uint32_t)dv;
+    }
+    ntt_fwd(x, S.d[r], S.twF, lane);
+#pragma unroll
+    for (int j = 0; j < 32; j++) S.d[r][kPadRow * lane + j] = red_2p(x[j]);
+    for (int m = 0; m < kParts; m++) {
+#pragma unroll
+        for (int j = 0; j < 32; j++) {
+            uint32_t v = polys[r * kN + lane + 32 * j];
+            const int32_t p0 = ((int32_t)((v & 0x7FFu) << 21)) >> 21;
+            v = (v - (uint32_t)p0) >> 11;
+            const int32_t p1 = ((int32_t)((v & 0x7FFu) << 21)) >> 21;
+            v = (v - (uint32_t)p1) >> 11;
+            const int32_t p2 = ((int32_t)((v & 0x3FFu) << 22)) >> 22;
+            const int32_t pm = m == 0 ? p0 : (m == 1 ? p1 : p2);
+            x[j] = pm < 0 ? (uint32_t)(pm + (int32_t)kP) : (uint32_t)pm;
+        }
+        ntt_fwd(x, S.b[r][m], S.twF, lane);
+#pragma unroll
+        for (int j = 0; j < 32; j++) S.b[r][m][kPadRow * lane + j] = red_p(shoup_mul(x[j], ninv, ninvp));
+    }
+    __syncthreads();
+    const uint32_t R = c_misc[0], Rp = c_misc[1];
+    for (int a = threadIdx.x; a < kN; a += blockDim.x) {
+        const int pa = a + (a >> 5);
+        for (int m = 0; m < kParts; m++) {
+            uint64_t acc = 0;
+            for (int rr = 0; rr < kRows; rr++) acc += (uint64_t)S.d[rr][pa] * S.b[rr][m][pa];
+            const uint32_t hi = (uint32_t)(acc >> 32), lo = (uint32_t)acc;
+            S.o[m][pa] = red_2p(shoup_mul(hi, R, Rp) + (lo - (lo >> 30) * kP));
+        }
+    }
+    __syncthreads();
+    if (r == 0) {
+        uint32_t sum[32];
+#pragma unroll
+        for (int j = 0; j < 32; j++) sum[j] = 0u;
+        for (int m = 0; m < kParts; m++) {
+#pragma unroll
+            for (int j = 0; j < 32; j++) x[j] = S.o[m][kPadRow * lane + j];
+            ntt_inv(x, S.o[m], S.twI, lane);
+#pragma unroll
+            for (int j = 0; j < 32; j++) sum[j] += lift_centred(x[j]) << (11 * m);
+        }
+#pragma unroll
+        for (int j = 0; j < 32; j++) res[lane + 32 * j] = sum[j];
+    }
+}
+
+int launch_ntt_muladd6(const int32_t* digits, const uint32_t* polys, uint32_t* res, const uint2* twF,
+                       const uint2* twI, uint32_t ninv, uint32_t ninvp, cudaStream_t st) {
+    const size_t smem = sizeof(DiagSmem);
+    if (cudaFuncSetAttribute(ntt_muladd6_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+        cudaSuccess)
+        return -1;
+    ntt_muladd6_kernel<<<1, 192, smem, st>>>(digits, polys, res, twF, twI, ninv, ninvp);
+    return 0;
+}
+
+// ---- microbenchmark: the kernels' own lazy CT butterfly and 64-bit MAC, register resident ----------
+template <int NV>
+__global__ void __launch_bounds__(256) mb_bfly_kernel(uint32_t* sink, int iters, uint32_t w, uint32_t wp) {
+    uint32_t x[NV], y[NV];
+#pragma unroll
+    for (int i = 0; i < NV; i++) {
+        x[i] = threadIdx.x * 7u + i;
+        y[i] = threadIdx.x * 13u + 3u * i;
+    }
+    for (int it = 0; it < iters; it++) {
+#pragma unroll
+        for (int i = 0; i < NV; i++) ct_bfly(x[i], y[i], w, wp);
+        w ^= (uint32_t)it & 1u;          // keep the twiddle loop-variant (uniform, cheap)
+    }
+    uint32_t s = 0;
+#pragma unroll
+    for (int i = 0; i < NV; i++) s += x[i] ^ y[i];
+    if (s == 0x12345678u) sink[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+template <int NV>
+__global__ void __launch_bounds__(256) mb_mac_kernel(uint64_t* sink, int iters, uint32_t b0) {
+    uint64_t acc[NV];
+    uint32_t d[NV];
+#pragma unroll
+    for (int i = 0; i < NV; i++) {
+        acc[i] = 0;
+        d[i] = threadIdx.x * 7u + i;
+    }
+    uint32_t b = b0 + threadIdx.x;
+    for (int it = 0; it < iters; it++) {
+#pragma unroll
+        for (int i = 0; i < NV; i++) acc[i] += (uint64_t)d[i] * b;
+        b += 3u;
+    }
+    uint64_t s = 0;
+#pragma unroll
+    for (int i = 0; i < NV; i++) s += acc[i];
+    if (s == 0x123456789ull) sink[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+
+int run_microbench(int iters, double* bfly, double* mac) {
+    int dev = 0, sms = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return -1;
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return -1;
+    const int blocks = sms * 8, threads = 256;
+    void* sink = nullptr;
+    if (cudaMalloc(&sink, (size_t)blocks * threads * 8) != cudaSuccess) return -1;
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    float best_b = 1e30f, best_m = 1e30f;
+    for (int rep = 0; rep < 4; rep++) {
+        float ms = 0;
+        cudaEventRecord(e0);
+        mb_bfly_kernel<16><<<blocks, threads>>>((uint32_t*)sink, iters, 123456789u, 987654u);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (rep > 0) best_b = ms < best_b ? ms : best_b;
+        cudaEventRecord(e0);
+        mb_mac_kernel<16><<<blocks, threads>>>((uint64_t*)sink, iters, 77u);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (rep > 0) best_m = ms < best_m ? ms : best_m;
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(sink);
+    if (cudaGetLastError() != cudaSuccess) return -1;
+    const double ops = (double)blocks * threads * iters * 16.0;
+    *bfly = ops / (best_b * 1e-3);
+    *mac = ops / (best_m * 1e-3);
+    return 0;
+}
+
+}  // namespace tb

@@ -1,0 +1,52 @@
+// tb_kernels.cuh -- kernel argument blocks and host launchers shared by the library's translation unit.
+#pragma once
+#include <cuda_runtime.h>
+
+#include "tb_common.cuh"
+
+namespace tb {
+
+// blind rotation + extraction over a batch of lanes (tb_bootstrap.cu)
+struct BrArgs {
+    const uint32_t* src0;
+    const uint32_t* src1;
+    const uint32_t* src2;
+    int64_t src_stride;        // words between ciphertext rows (>= n + 1)
+    const LaneDesc* lanes;
+    int32_t nlanes;
+    const uint32_t* bkhat;     // [n][6 rows][6 outs][N]  (u32 < p)
+    const uint2* twF;          // [31][32] per-lane forward twiddles (w, w')
+    const uint2* twI;          // [31][32] per-lane inverse twiddles
+    uint32_t* out;             // [nlanes][out_stride] extracted LWE(N) samples
+    int64_t out_stride;        // words between output rows (>= N + 1; kLaneStride for the lane buffer)
+};
+
+// key switch + MUX combine + NOT over a batch of gates (tb_keyswitch.cu)
+struct KsArgs {
+    const uint32_t* lanes;      // extracted samples from br_kernel
+    int32_t lane_base;          // GateDesc.lane* - lane_base = row in `lanes`
+    int64_t lane_stride;        // words between lane rows (kLaneStride for the lane buffer)
+    const GateDesc* gates;
+    int32_t ngates;
+    const uint32_t* ksk;        // [N][t][3][kKsRow]  (digit-0 rows dropped)
+    uint32_t* out;              // output ciphertext rows
+    int64_t out_stride;
+    const uint32_t* not_src;    // NOT input rows
+    int64_t not_stride;
+};
+
+int launch_br(const BrArgs& A, int G, cudaStream_t st);
+size_t br_smem_bytes(int G);
+void launch_bk_to_ntt(const uint32_t* bk, uint32_t* bkhat, const uint2* twF, uint32_t ninv, uint32_t ninvp,
+                      cudaStream_t st);
+void launch_build_gate_desc(int kind, int32_t wa, int32_t wb, uint32_t cst, int64_t count, LaneDesc* lanes,
+                            GateDesc* gates, cudaStream_t st);
+int launch_ks(const KsArgs& A, cudaStream_t st);
+void launch_ksk_relayout(const uint32_t* src, uint32_t* dst, cudaStream_t st);
+int set_ntt_constants(const uint32_t* fw, const uint32_t* fwp, const uint32_t* iw, const uint32_t* iwp,
+                      const uint32_t* misc);
+int launch_ntt_muladd6(const int32_t* digits, const uint32_t* polys, uint32_t* res, const uint2* twF,
+                       const uint2* twI, uint32_t ninv, uint32_t ninvp, cudaStream_t st);
+int run_microbench(int iters, double* bfly, double* mac);
+
+}  // namespace tb

@@ -1,0 +1,118 @@
+// tb_keyswitch.cu -- batched LWE key switching N -> n ("key switching", the second slice
+// of a gate's profile, Fig. 7, named as vectorisable at P:247), plus the MUX lane combine and
+// NOT (negation, no bootstrap) of a level.
+//
+// out = (0, b) - sum_{i < N, j < t, d_ij != 0} KSK[i][j][d_ij], d_ij = base-4 digits of a_i + 2^15 (C9).
+// A CTA owns a tile of T gates; its threads own 4 consecutive output words each (16-B vector loads of the
+// 632-word device KSK rows).  For every (i, j) the digits of the T gates select rows of the 3-row group
+// KSK[i][j][1..3]; the group is read from L2 once per tile and re-read from L1 by the other gates, so HBM/L2
+// traffic per gate is (62 MB KSK) / T instead of 15.5 MB of data-dependent row gathers.
+#include "tb_kernels.cuh"
+
+namespace tb {
+
+constexpr int kKsThreads = 160;                  // 158 threads x 4 words = 632 words
+
+template <int T>
+__global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A) {
+    __shared__ __align__(16) uint16_t sW[kN][T];  // (a_i + 2^15) >> 16: all 8 digits of a_i
+    __shared__ uint32_t sB[T];
+    const int tid = threadIdx.x;
+    const int g0 = blockIdx.x * T;
+
+    // prologue: combine lanes (MUX: u1 + u2 + (0, mu)), take digit words
+    for (int g = 0; g < T; g++) {
+        const int gi = g0 + g;
+        GateDesc gd = {0, 0, -1, kGateNot};
+        bool valid = gi < A.ngates;
+        if (valid) gd = A.gates[gi];
+        const bool boot = valid && gd.kind != kGateNot;
+        const uint32_t* l0 = A.lanes + (int64_t)(gd.lane0 - A.lane_base) * A.lane_stride;
+        const uint32_t* l1 = gd.lane1 >= 0 ? A.lanes + (int64_t)(gd.lane1 - A.lane_base) * A.lane_stride : nullptr;
+        for (int i = tid; i <= kN; i += kKsThreads) {
+            uint32_t e = 0u;
+            if (boot) {
+                e = __ldg(l0 + i);
+                if (l1) e += __ldg(l1 + i);
+            }
+            if (i < kN) sW[i][g] = boot ? (uint16_t)((e + (1u << 15)) >> 16) : (uint16_t)0;
+            else sB[g] = l1 ? e + kMu : e;
+        }
+    }
+    __syncthreads();
+
+    const int k0 = 4 * tid;                         // output words k0..k0+3
+    const bool active = tid < kKsRow / 4;
+    uint32_t acc[T][4];
+#pragma unroll
+    for (int g = 0; g < T; g++) {
+        const int gi = g0 + g;
+        const bool isnot = gi < A.ngates && A.gates[gi].kind == kGateNot;
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            const int k = k0 + q;
+            uint32_t v = (k == kn) ? sB[g] : 0u;
+            if (isnot && active && k <= kn) v = 0u - __ldg(A.not_src + (int64_t)A.gates[gi].lane0 * A.not_stride + k);
+            acc[g][q] = v;
+        }
+    }
+    if (active) {
+        for (int i = 0; i < kN; i++) {
+            uint16_t w[T];
+#pragma unroll
+            for (int g = 0; g < T; g += 8) {
+                const uint4 v = *reinterpret_cast<const uint4*>(&sW[i][g]);
+                w[g + 0] = (uint16_t)(v.x & 0xFFFF); w[g + 1] = (uint16_t)(v.x >> 16);
+                w[g + 2] = (uint16_t)(v.y & 0xFFFF); w[g + 3] = (uint16_t)(v.y >> 16);
+                w[g + 4] = (uint16_t)(v.z & 0xFFFF); w[g + 5] = (uint16_t)(v.z >> 16);
+                w[g + 6] = (uint16_t)(v.w & 0xFFFF); w[g + 7] = (uint16_t)(v.w >> 16);
+            }
+            const uint32_t* rowi = A.ksk + (size_t)i * kKsT * (kKsBase - 1) * kKsRow + k0;
+#pragma unroll
+            for (int j = 0; j < kKsT; j++) {
+#pragma unroll
+                for (int g = 0; g < T; g++) {
+                    const uint32_t d = (w[g] >> (14 - 2 * j)) & 3u;
+                    if (d) {
+                        const uint4 v = __ldg(reinterpret_cast<const uint4*>(rowi + (j * (kKsBase - 1) + d - 1) * kKsRow));
+                        acc[g][0] -= v.x; acc[g][1] -= v.y; acc[g][2] -= v.z; acc[g][3] -= v.w;
+                    }
+                }
+            }
+        }
+#pragma unroll
+        for (int g = 0; g < T; g++) {
+            const int gi = g0 + g;
+            if (gi < A.ngates) {
+                uint32_t* o = A.out + (int64_t)A.gates[gi].out_row * A.out_stride;
+#pragma unroll
+                for (int q = 0; q < 4; q++)
+                    if (k0 + q <= kn) o[k0 + q] = acc[g][q];
+            }
+        }
+    }
+}
+
+// digit-0 rows dropped, rows padded to 632 words: [i][j][d][631] (host layout) -> [i][j][d-1][632]
+__global__ void ksk_relayout_kernel(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst) {
+    const size_t row = blockIdx.x;                   // (i, j, d-1)
+    const size_t dm1 = row % (kKsBase - 1), ij = row / (kKsBase - 1);
+    const uint32_t* s = src + (ij * kKsBase + dm1 + 1) * (kn + 1);
+    uint32_t* d = dst + row * kKsRow;
+    for (int k = threadIdx.x; k < kKsRow; k += blockDim.x) d[k] = k <= kn ? s[k] : 0u;
+}
+
+constexpr int kKsTile = 16;
+
+int launch_ks(const KsArgs& A, cudaStream_t st) {
+    if (A.ngates <= 0) return 0;
+    const int blocks = (A.ngates + kKsTile - 1) / kKsTile;
+    ks_kernel<kKsTile><<<blocks, kKsThreads, 0, st>>>(A);
+    return 0;
+}
+
+void launch_ksk_relayout(const uint32_t* src, uint32_t* dst, cudaStream_t st) {
+    ksk_relayout_kernel<<<kN * kKsT * (kKsBase - 1), 128, 0, st>>>(src, dst);
+}
+
+}  // namespace tb

@@ -1,0 +1,622 @@
+// tb_runtime.cu -- the C ABI (include/tfhe_b200.h): contexts, key upload, batched gates, Algorithm-1
+// levelisation and the level executor.  Host-side C++17; every arithmetic step of a gate runs in the
+// kernels of tb_bootstrap.cu / tb_keyswitch.cu.  There is no CPU fallback: without a usable sm_100 device
+// every entry point fails with an error status.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/tfhe_b200.h"
+#include "tb_kernels.cuh"
+
+
+using namespace tb;
+
+// ------------------------------------------------------------------------------------------ errors
+static thread_local std::string g_err;
+static int fail(int code, const char* msg) {
+    g_err = msg;
+    return code;
+}
+static int cuda_fail(cudaError_t e, const char* where) {
+    g_err = std::string(where) + ": " + cudaGetErrorString(e);
+    return TB_ECUDA;
+}
+#define TB_CUDA(call)                                            \
+    do {                                                         \
+        cudaError_t e_ = (call);                                 \
+        if (e_ != cudaSuccess) return cuda_fail(e_, #call);      \
+    } while (0)
+
+extern "C" const char* tb_last_error(void) { return g_err.c_str(); }
+extern "C" const char* tb_version(void) { return "tfhe_b200 0.1 (sm_100a; n=630 N=1024 l=3 Bgbit=7 t=8 base=4)"; }
+
+// ------------------------------------------------------------------------------------------ field setup
+static uint32_t mulmod(uint64_t a, uint64_t b) { return (uint32_t)((a * b) % kP); }
+static uint32_t powmod(uint64_t b, uint64_t e) {
+    uint64_t r = 1;
+    b %= kP;
+    while (e) {
+        if (e & 1) r = r * b % kP;
+        b = b * b % kP;
+        e >>= 1;
+    }
+    return (uint32_t)r;
+}
+static uint32_t shoup_of(uint32_t w) { return (uint32_t)(((uint64_t)w << 32) / kP); }
+static uint32_t brv10(uint32_t k) {
+    uint32_t r = 0;
+    for (int b = 0; b < 10; b++) r |= ((k >> b) & 1u) << (9 - b);
+    return r;
+}
+
+struct tb_ctx {
+    int device = 0;
+    int lanes_per_cta = 2;
+    cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
+    uint2* twF = nullptr;                   // [31][32]
+    uint2* twI = nullptr;
+    uint32_t ninv = 0, ninvp = 0;
+    uint32_t* bkhat = nullptr;              // [n][6][6][N]
+    uint32_t* ksk = nullptr;                // [N][t][3][632]
+    bool have_bk = false, have_ksk = false;
+    // scratch (grown on demand; growing synchronises the device)
+    uint32_t* lanebuf = nullptr;
+    int64_t lanebuf_rows = 0;
+    LaneDesc* ldesc = nullptr;
+    GateDesc* gdesc = nullptr;
+    int64_t desc_rows = 0;
+    uint32_t* stage = nullptr;              // tb_gates_host staging
+    size_t stage_words = 0;
+};
+
+struct tb_dev_netlist {
+    int64_t n_inputs = 0, n_gates = 0, n_levels = 0;
+    std::vector<int64_t> level_off;         // [n_levels + 1] gate offsets (level-sorted order)
+    std::vector<int64_t> lane_off;          // [n_gates + 1] lane prefix over level-sorted gates
+    std::vector<int64_t> boot_prefix;       // [n_gates + 1] bootstrapped gates (non-NOT) prefix
+    std::vector<int64_t> row_of_wire;       // [n_inputs + n_gates]
+    LaneDesc* ldesc = nullptr;
+    GateDesc* gdesc = nullptr;
+};
+
+static int grow_lanes(tb_ctx* c, int64_t rows) {
+    if (rows <= c->lanebuf_rows) return TB_OK;
+    int64_t want = std::max<int64_t>(rows, c->lanebuf_rows * 3 / 2);
+    if (c->lanebuf) cudaFree(c->lanebuf);
+    c->lanebuf = nullptr;
+    c->lanebuf_rows = 0;
+    if (cudaMalloc(&c->lanebuf, (size_t)want * kLaneStride * 4) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(TB_ENOMEM, "lane buffer allocation failed");
+    }
+    c->lanebuf_rows = want;
+    return TB_OK;
+}
+static int grow_desc(tb_ctx* c, int64_t rows) {
+    if (rows <= c->desc_rows) return TB_OK;
+    int64_t want = std::max<int64_t>(rows, c->desc_rows * 3 / 2);
+    if (c->ldesc) cudaFree(c->ldesc);
+    if (c->gdesc) cudaFree(c->gdesc);
+    c->ldesc = nullptr;
+    c->gdesc = nullptr;
+    c->desc_rows = 0;
+    if (cudaMalloc(&c->ldesc, (size_t)want * 2 * sizeof(LaneDesc)) != cudaSuccess ||
+        cudaMalloc(&c->gdesc, (size_t)want * sizeof(GateDesc)) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(TB_ENOMEM, "descriptor allocation failed");
+    }
+    c->desc_rows = want;
+    return TB_OK;
+}
+
+extern "C" tb_params tb_default_params(void) {
+    tb_params p;
+    p.n = kn; p.N = kN; p.k = 1; p.l = kL; p.Bgbit = kBgbit; p.ks_t = kKsT; p.ks_basebit = kKsBasebit;
+    return p;
+}
+
+extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
+    if (!P || !out) return fail(TB_EINVAL, "null argument");
+    *out = nullptr;
+    if (P->n != kn || P->N != kN || P->k != 1 || P->l != kL || P->Bgbit != kBgbit || P->ks_t != kKsT ||
+        P->ks_basebit != kKsBasebit)
+        return fail(TB_EUNSUPPORTED, "only n=630 N=1024 k=1 l=3 Bgbit=7 ks_t=8 ks_basebit=2 is compiled");
+    int ndev = 0;
+    TB_CUDA(cudaGetDeviceCount(&ndev));
+    if (dev < 0 || dev >= ndev) return fail(TB_EINVAL, "bad device index");
+    cudaDeviceProp prop;
+    TB_CUDA(cudaGetDeviceProperties(&prop, dev));
+    if (prop.major != 10 || prop.minor != 0) return fail(TB_EUNSUPPORTED, "device is not sm_100 (B200)");
+    TB_CUDA(cudaSetDevice(dev));
+    tb_ctx* c = new (std::nothrow) tb_ctx();
+    if (!c) return fail(TB_ENOMEM, "host allocation failed");
+    c->device = dev;
+
+    // psi: primitive 2N-th root of unity mod p (psi^N = -1)
+    uint32_t psi = 0;
+    for (uint32_t g = 2; g < 1000 && !psi; g++) {
+        uint32_t cand = powmod(g, (kP - 1) / kTwoN);
+        if (powmod(cand, kN) == kP - 1) psi = cand;
+    }
+    const uint32_t psi_inv = powmod(psi, kP - 2);
+    uint32_t fw[32] = {0}, fwp[32] = {0}, iw[32] = {0}, iwp[32] = {0}, misc[4] = {0};
+    for (uint32_t k = 1; k < 32; k++) {
+        fw[k] = powmod(psi, brv10(k));
+        iw[k] = powmod(psi_inv, brv10(k));
+        fwp[k] = shoup_of(fw[k]);
+        iwp[k] = shoup_of(iw[k]);
+    }
+    misc[0] = (uint32_t)((1ull << 32) % kP);
+    misc[1] = shoup_of(misc[0]);
+    std::vector<uint2> tf(31 * 32), ti(31 * 32);
+    for (int s = 5; s < 10; s++)
+        for (int bj = 0; bj < (1 << (s - 5)); bj++)
+            for (int t = 0; t < 32; t++) {
+                const uint32_t k = (1u << s) + (uint32_t)t * (1u << (s - 5)) + bj;
+                const int e = (1 << (s - 5)) - 1 + bj;
+                const uint32_t w = powmod(psi, brv10(k)), wi = powmod(psi_inv, brv10(k));
+                tf[e * 32 + t] = make_uint2(w, shoup_of(w));
+                ti[e * 32 + t] = make_uint2(wi, shoup_of(wi));
+            }
+    c->ninv = powmod(kN, kP - 2);
+    c->ninvp = shoup_of(c->ninv);
+    int rc = set_ntt_constants(fw, fwp, iw, iwp, misc);
+    cudaError_t e = cudaSuccess;
+    if (rc == 0) e = cudaStreamCreateWithFlags(&c->own, cudaStreamNonBlocking);
+    if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->twF, 31 * 32 * sizeof(uint2));
+    if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->twI, 31 * 32 * sizeof(uint2));
+    if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->twF, tf.data(), tf.size() * sizeof(uint2), cudaMemcpyHostToDevice);
+    if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->twI, ti.data(), ti.size() * sizeof(uint2), cudaMemcpyHostToDevice);
+    if (rc != 0 || e != cudaSuccess) {
+        tb_ctx_destroy(c);
+        return e != cudaSuccess ? cuda_fail(e, "tb_ctx_create") : fail(TB_ECUDA, "constant upload failed");
+    }
+    *out = c;
+    return TB_OK;
+}
+
+extern "C" int tb_ctx_destroy(tb_ctx* c) {
+    if (!c) return TB_OK;
+    cudaSetDevice(c->device);
+    cudaFree(c->twF);
+    cudaFree(c->twI);
+    cudaFree(c->bkhat);
+    cudaFree(c->ksk);
+    cudaFree(c->lanebuf);
+    cudaFree(c->ldesc);
+    cudaFree(c->gdesc);
+    cudaFree(c->stage);
+    if (c->own) cudaStreamDestroy(c->own);
+    delete c;
+    return TB_OK;
+}
+
+extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
+    if (!c || lanes < 1 || lanes > 4) return fail(TB_EINVAL, "lanes per CTA must be 1..4");
+    c->lanes_per_cta = lanes;
+    return TB_OK;
+}
+
+extern "C" int tb_key_bytes(const tb_ctx* c, size_t* bytes) {
+    if (!c || !bytes) return fail(TB_EINVAL, "null argument");
+    *bytes = (c->have_bk ? (size_t)kn * kRows * kOuts * kN * 4 : 0) +
+             (c->have_ksk ? (size_t)kN * kKsT * (kKsBase - 1) * kKsRow * 4 : 0);
+    return TB_OK;
+}
+
+extern "C" int tb_load_bk(tb_ctx* c, const uint32_t* host_bk, size_t n_words) {
+    if (!c || !host_bk) return fail(TB_EINVAL, "null argument");
+    const size_t want = (size_t)kn * kRows * 2 * kN;
+    if (n_words != want) return fail(TB_EINVAL, "bootstrapping key must have n*2l*2*N words");
+    TB_CUDA(cudaSetDevice(c->device));
+    if (!c->bkhat) TB_CUDA(cudaMalloc(&c->bkhat, (size_t)kn * kRows * kOuts * kN * 4));
+    uint32_t* tmp = nullptr;
+    TB_CUDA(cudaMalloc(&tmp, want * 4));
+    cudaError_t e = cudaMemcpyAsync(tmp, host_bk, want * 4, cudaMemcpyHostToDevice, c->own);
+    if (e == cudaSuccess) {
+        launch_bk_to_ntt(tmp, c->bkhat, c->twF, c->ninv, c->ninvp, c->own);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(c->own);
+    cudaFree(tmp);
+    if (e != cudaSuccess) return cuda_fail(e, "tb_load_bk");
+    c->have_bk = true;
+    return TB_OK;
+}
+
+extern "C" int tb_load_ksk(tb_ctx* c, const uint32_t* host_ksk, size_t n_words) {
+    if (!c || !host_ksk) return fail(TB_EINVAL, "null argument");
+    const size_t want = (size_t)kN * kKsT * kKsBase * (kn + 1);
+    if (n_words != want) return fail(TB_EINVAL, "key-switching key must have N*t*base*(n+1) words");
+    TB_CUDA(cudaSetDevice(c->device));
+    if (!c->ksk) TB_CUDA(cudaMalloc(&c->ksk, (size_t)kN * kKsT * (kKsBase - 1) * kKsRow * 4));
+    uint32_t* tmp = nullptr;
+    TB_CUDA(cudaMalloc(&tmp, want * 4));
+    cudaError_t e = cudaMemcpyAsync(tmp, host_ksk, want * 4, cudaMemcpyHostToDevice, c->own);
+    if (e == cudaSuccess) {
+        launch_ksk_relayout(tmp, c->ksk, c->own);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(c->own);
+    cudaFree(tmp);
+    if (e != cudaSuccess) return cuda_fail(e, "tb_load_ksk");
+    c->have_ksk = true;
+    return TB_OK;
+}
+
+// ------------------------------------------------------------------------------------------ gates
+// (C_g, w_a, w_b) per two-input gate: tfhe-lib's bootstrapped gates (EXT[10]; SURVEY 8(c) gate table)
+static bool gate_linear(int gate, uint32_t* C, int32_t* wa, int32_t* wb) {
+    const uint32_t e8 = kMu, e4 = 2u * kMu;
+    switch (gate) {
+        case TB_NAND:  *C = e8;      *wa = -1; *wb = -1; return true;
+        case TB_AND:   *C = 0u - e8; *wa = 1;  *wb = 1;  return true;
+        case TB_OR:    *C = e8;      *wa = 1;  *wb = 1;  return true;
+        case TB_NOR:   *C = 0u - e8; *wa = -1; *wb = -1; return true;
+        case TB_XOR:   *C = e4;      *wa = 2;  *wb = 2;  return true;
+        case TB_XNOR:  *C = 0u - e4; *wa = -2; *wb = -2; return true;
+        case TB_ANDNY: *C = 0u - e8; *wa = -1; *wb = 1;  return true;
+        case TB_ANDYN: *C = 0u - e8; *wa = 1;  *wb = -1; return true;
+        case TB_ORNY:  *C = e8;      *wa = -1; *wb = 1;  return true;
+        case TB_ORYN:  *C = e8;      *wa = 1;  *wb = -1; return true;
+        default: return false;
+    }
+}
+static bool gate_known(int g) {
+    uint32_t C; int32_t a, b;
+    return g == TB_NOT || g == TB_MUX || gate_linear(g, &C, &a, &b);
+}
+
+static int check_ready(tb_ctx* c) {
+    if (!c) return fail(TB_EINVAL, "null context");
+    if (!c->have_bk || !c->have_ksk) return fail(TB_ENOKEYS, "load the bootstrapping and key-switching keys first");
+    return TB_OK;
+}
+
+static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint32_t* s2, int64_t sstride,
+                  const LaneDesc* lanes, int64_t nlanes, uint32_t* out, int64_t ostride, cudaStream_t st) {
+    if (nlanes <= 0) return TB_OK;
+    BrArgs A;
+    A.src0 = s0; A.src1 = s1; A.src2 = s2; A.src_stride = sstride;
+    A.lanes = lanes; A.nlanes = (int32_t)nlanes; A.bkhat = c->bkhat; A.twF = c->twF; A.twI = c->twI;
+    A.out = out; A.out_stride = ostride;
+    int rc = launch_br(A, c->lanes_per_cta, st);
+    if (rc) return fail(TB_ECUDA, "blind-rotation kernel attribute/launch failed");
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "br_kernel launch");
+    return TB_OK;
+}
+static int run_ks(tb_ctx* c, const uint32_t* lanes, int64_t lane_base, int64_t lane_stride, const GateDesc* gates,
+                  int64_t ngates, uint32_t* out, int64_t ostride, const uint32_t* not_src, int64_t not_stride,
+                  cudaStream_t st) {
+    if (ngates <= 0) return TB_OK;
+    KsArgs A;
+    A.lanes = lanes; A.lane_base = (int32_t)lane_base; A.lane_stride = lane_stride; A.gates = gates;
+    A.ngates = (int32_t)ngates; A.ksk = c->ksk; A.out = out; A.out_stride = ostride; A.not_src = not_src;
+    A.not_stride = not_stride;
+    launch_ks(A, st);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "ks_kernel launch");
+    return TB_OK;
+}
+
+extern "C" int tb_gates(tb_ctx* c, int gate, const uint32_t* ca, const uint32_t* cb, const uint32_t* cc,
+                        uint32_t* out, int64_t count, int64_t stride, tb_stream stream) {
+    int rc = check_ready(c);
+    if (rc) return rc;
+    if (count < 0 || stride < kn + 1 || count > (int64_t)1 << 30) return fail(TB_EINVAL, "bad count or stride");
+    if (!gate_known(gate)) return fail(TB_EINVAL, "unknown gate code");
+    if (count == 0) return TB_OK;
+    if (!ca || !out || (gate != TB_NOT && !cb) || (gate == TB_MUX && !cc)) return fail(TB_EINVAL, "null array");
+    TB_CUDA(cudaSetDevice(c->device));
+    cudaStream_t st = (cudaStream_t)stream;
+    const int64_t nl = gate == TB_MUX ? 2 * count : (gate == TB_NOT ? 0 : count);
+    if ((rc = grow_desc(c, count))) return rc;
+    if ((rc = grow_lanes(c, std::max<int64_t>(nl, 1)))) return rc;
+    uint32_t C = 0; int32_t wa = 0, wb = 0;
+    gate_linear(gate, &C, &wa, &wb);
+    const int kind = gate == TB_NOT ? kGateNot : (gate == TB_MUX ? kGateMux : kGateBoot);
+    launch_build_gate_desc(kind, wa, wb, C, count, c->ldesc, c->gdesc, st);
+    if ((rc = run_br(c, ca, cb, cc, stride, c->ldesc, nl, c->lanebuf, kLaneStride, st))) return rc;
+    return run_ks(c, c->lanebuf, 0, kLaneStride, c->gdesc, count, out, stride, ca, stride, st);
+}
+
+extern "C" int tb_gates_host(tb_ctx* c, int gate, const uint32_t* hca, const uint32_t* hcb, const uint32_t* hcc,
+                             uint32_t* hout, int64_t count, int64_t stride) {
+    int rc = check_ready(c);
+    if (rc) return rc;
+    if (count < 0 || stride < kn + 1) return fail(TB_EINVAL, "bad count or stride");
+    if (!gate_known(gate)) return fail(TB_EINVAL, "unknown gate code");
+    if (count == 0) return TB_OK;
+    if (!hca || !hout || (gate != TB_NOT && !hcb) || (gate == TB_MUX && !hcc)) return fail(TB_EINVAL, "null array");
+    TB_CUDA(cudaSetDevice(c->device));
+    const size_t words = (size_t)count * stride;
+    if (c->stage_words < 4 * words) {
+        cudaFree(c->stage);
+        c->stage = nullptr;
+        c->stage_words = 0;
+        if (cudaMalloc(&c->stage, 4 * words * 4) != cudaSuccess) {
+            cudaGetLastError();
+            return fail(TB_ENOMEM, "staging allocation failed");
+        }
+        c->stage_words = 4 * words;
+    }
+    uint32_t *da = c->stage, *db = c->stage + words, *dc = c->stage + 2 * words, *dout = c->stage + 3 * words;
+    TB_CUDA(cudaMemcpyAsync(da, hca, words * 4, cudaMemcpyHostToDevice, c->own));
+    if (gate != TB_NOT) TB_CUDA(cudaMemcpyAsync(db, hcb, words * 4, cudaMemcpyHostToDevice, c->own));
+    if (gate == TB_MUX) TB_CUDA(cudaMemcpyAsync(dc, hcc, words * 4, cudaMemcpyHostToDevice, c->own));
+    rc = tb_gates(c, gate, da, db, dc, dout, count, stride, (tb_stream)c->own);
+    if (rc) return rc;
+    TB_CUDA(cudaMemcpyAsync(hout, dout, words * 4, cudaMemcpyDeviceToHost, c->own));
+    TB_CUDA(cudaStreamSynchronize(c->own));
+    return TB_OK;
+}
+
+extern "C" int tb_bootstrap_wo_ks(tb_ctx* c, const uint32_t* in, int64_t in_stride, uint32_t* out,
+                                  int64_t out_stride, int64_t count, tb_stream stream) {
+    if (!c) return fail(TB_EINVAL, "null context");
+    if (!c->have_bk) return fail(TB_ENOKEYS, "load the bootstrapping key first");
+    if (count < 0 || in_stride < kn + 1 || out_stride < kN + 1) return fail(TB_EINVAL, "bad count or stride");
+    if (count == 0) return TB_OK;
+    if (!in || !out) return fail(TB_EINVAL, "null array");
+    TB_CUDA(cudaSetDevice(c->device));
+    int rc = grow_desc(c, count);
+    if (rc) return rc;
+    cudaStream_t st = (cudaStream_t)stream;
+    launch_build_gate_desc(kGateBoot, 1, 0, 0u, count, c->ldesc, c->gdesc, st);
+    return run_br(c, in, in, in, in_stride, c->ldesc, count, out, out_stride, st);
+}
+
+extern "C" int tb_keyswitch(tb_ctx* c, const uint32_t* in, int64_t in_stride, uint32_t* out, int64_t out_stride,
+                            int64_t count, tb_stream stream) {
+    if (!c) return fail(TB_EINVAL, "null context");
+    if (!c->have_ksk) return fail(TB_ENOKEYS, "load the key-switching key first");
+    if (count < 0 || in_stride < kN + 1 || out_stride < kn + 1) return fail(TB_EINVAL, "bad count or stride");
+    if (count == 0) return TB_OK;
+    if (!in || !out) return fail(TB_EINVAL, "null array");
+    TB_CUDA(cudaSetDevice(c->device));
+    int rc = grow_desc(c, count);
+    if (rc) return rc;
+    cudaStream_t st = (cudaStream_t)stream;
+    launch_build_gate_desc(kGateBoot, 1, 0, 0u, count, c->ldesc, c->gdesc, st);
+    return run_ks(c, in, 0, in_stride, c->gdesc, count, out, out_stride, in, in_stride, st);
+}
+
+extern "C" int tb_ntt_muladd6(tb_ctx* c, const int32_t* digits, const uint32_t* polys, uint32_t* res) {
+    if (!c || !digits || !polys || !res) return fail(TB_EINVAL, "null argument");
+    TB_CUDA(cudaSetDevice(c->device));
+    if (launch_ntt_muladd6(digits, polys, res, c->twF, c->twI, c->ninv, c->ninvp, c->own))
+        return fail(TB_ECUDA, "ntt_muladd6 launch failed");
+    TB_CUDA(cudaGetLastError());
+    TB_CUDA(cudaStreamSynchronize(c->own));
+    return TB_OK;
+}
+
+extern "C" int tb_microbench(tb_ctx* c, int iters, double* bfly, double* mac) {
+    if (!c || !bfly || !mac || iters <= 0) return fail(TB_EINVAL, "bad argument");
+    TB_CUDA(cudaSetDevice(c->device));
+    if (run_microbench(iters, bfly, mac)) return fail(TB_ECUDA, "microbenchmark failed");
+    return TB_OK;
+}
+
+// ------------------------------------------------------------------------------------------ netlists
+// Algorithm 1: starting from the inputs (ready = finished = I), each iteration computes every
+// node whose predecessors are all ready.  The iteration in which gate g first enters C - finished is
+// 1 + max(level of its predecessors) (inputs = level 0), computed here with one Kahn pass (C14: k = 1).
+static int levelise_impl(const tb_netlist* net, std::vector<int64_t>& level, int64_t* n_levels) {
+    if (!net || net->n_inputs < 0 || net->n_gates < 0) return fail(TB_EINVAL, "bad netlist");
+    const int64_t ni = net->n_inputs, ng = net->n_gates, nw = ni + ng;
+    if (ng > 0 && (!net->type || !net->in0 || !net->in1)) return fail(TB_EINVAL, "null netlist array");
+    level.assign((size_t)ng, -1);
+    std::vector<int32_t> pending((size_t)ng, 0);
+    std::vector<int64_t> head((size_t)nw + 1, 0), adj;
+    auto ins = [&](int64_t g, int64_t k) -> int64_t {
+        if (k == 0) return net->in0[g];
+        if (k == 1) return net->type[g] == TB_NOT ? -1 : net->in1[g];
+        return (net->type[g] == TB_MUX && net->in2) ? net->in2[g] : -1;
+    };
+    for (int64_t g = 0; g < ng; g++) {
+        const int t = net->type[g];
+        if (!gate_known(t)) return fail(TB_EINVAL, "unknown gate code in netlist");
+        for (int k = 0; k < 3; k++) {
+            const int64_t w = ins(g, k);
+            const bool needed = k == 0 || (k == 1 && t != TB_NOT) || (k == 2 && t == TB_MUX);
+            if (!needed) continue;
+            if (w < 0 || w >= nw) return fail(TB_EINVAL, "wire index out of range");
+            if (w == ni + g) return fail(TB_EINVAL, "gate reads its own output (cycle)");
+            if (w >= ni) {
+                pending[g]++;
+                head[w + 1]++;
+            }
+        }
+    }
+    for (int64_t w = 0; w < nw; w++) head[w + 1] += head[w];
+    adj.resize((size_t)head[nw]);
+    std::vector<int64_t> fill(head.begin(), head.end() - 1);
+    for (int64_t g = 0; g < ng; g++) {
+        const int t = net->type[g];
+        for (int k = 0; k < 3; k++) {
+            const bool needed = k == 0 || (k == 1 && t != TB_NOT) || (k == 2 && t == TB_MUX);
+            if (!needed) continue;
+            const int64_t w = ins(g, k);
+            if (w >= ni) adj[fill[w]++] = g;
+        }
+    }
+    std::vector<int64_t> ready;                 // the current C - finished frontier
+    for (int64_t g = 0; g < ng; g++)
+        if (pending[g] == 0) { level[g] = 1; ready.push_back(g); }
+    int64_t done = 0, L = ready.empty() ? 0 : 1;
+    std::vector<int64_t> next;
+    while (!ready.empty()) {
+        next.clear();
+        for (int64_t g : ready) {
+            done++;
+            const int64_t w = ni + g;
+            for (int64_t e = head[w]; e < head[w + 1]; e++) {
+                const int64_t h = adj[e];
+                if (--pending[h] == 0) { level[h] = L + 1; next.push_back(h); }
+            }
+        }
+        if (!next.empty()) L++;
+        ready.swap(next);
+    }
+    if (done != ng) return fail(TB_EINVAL, "netlist has a cycle");
+    *n_levels = L;
+    return TB_OK;
+}
+
+extern "C" int tb_levelise(const tb_netlist* net, int64_t* level_of_gate, int64_t* n_levels) {
+    if (!level_of_gate || !n_levels) return fail(TB_EINVAL, "null argument");
+    std::vector<int64_t> lv;
+    int rc = levelise_impl(net, lv, n_levels);
+    if (rc) return rc;
+    std::copy(lv.begin(), lv.end(), level_of_gate);
+    return TB_OK;
+}
+
+extern "C" int tb_netlist_upload(tb_ctx* c, const tb_netlist* net, tb_dev_netlist** out) {
+    if (!c || !net || !out) return fail(TB_EINVAL, "null argument");
+    *out = nullptr;
+    std::vector<int64_t> lv;
+    int64_t nlev = 0;
+    int rc = levelise_impl(net, lv, &nlev);
+    if (rc) return rc;
+    const int64_t ni = net->n_inputs, ng = net->n_gates;
+    if (ni + ng > INT32_MAX) return fail(TB_EINVAL, "netlist too large for 32-bit rows");
+    tb_dev_netlist* d = new (std::nothrow) tb_dev_netlist();
+    if (!d) return fail(TB_ENOMEM, "host allocation failed");
+    d->n_inputs = ni; d->n_gates = ng; d->n_levels = nlev;
+    // counting sort by level (stable: ascending original index inside a level)
+    d->level_off.assign((size_t)nlev + 2, 0);
+    for (int64_t g = 0; g < ng; g++) d->level_off[lv[g]]++;
+    {
+        int64_t s = 0;
+        for (int64_t L = 1; L <= nlev; L++) { int64_t k = d->level_off[L]; d->level_off[L] = s; s += k; }
+        d->level_off[nlev + 1] = s;
+    }
+    std::vector<int64_t> order((size_t)ng), pos(d->level_off.begin(), d->level_off.end());
+    for (int64_t g = 0; g < ng; g++) order[pos[lv[g]]++] = g;
+    // level_off[L] (1-based) -> store 0-based [n_levels + 1]
+    std::vector<int64_t> lo((size_t)nlev + 1);
+    for (int64_t L = 0; L <= nlev; L++) lo[L] = d->level_off[L + 1];
+    d->level_off.swap(lo);
+    d->row_of_wire.resize((size_t)(ni + ng));
+    for (int64_t w = 0; w < ni; w++) d->row_of_wire[w] = w;
+    for (int64_t k = 0; k < ng; k++) d->row_of_wire[ni + order[k]] = ni + k;
+    // descriptors in level-sorted order
+    std::vector<GateDesc> gd((size_t)ng);
+    std::vector<LaneDesc> ld;
+    ld.reserve((size_t)ng);
+    d->lane_off.assign((size_t)ng + 1, 0);
+    d->boot_prefix.assign((size_t)ng + 1, 0);
+    for (int64_t k = 0; k < ng; k++) {
+        const int64_t g = order[k];
+        const int t = net->type[g];
+        const int32_t ra = (int32_t)d->row_of_wire[net->in0[g]];
+        GateDesc G;
+        G.out_row = (int32_t)(ni + k);
+        G.lane1 = -1;
+        if (t == TB_NOT) {
+            G.kind = kGateNot;
+            G.lane0 = ra;
+        } else if (t == TB_MUX) {
+            const int32_t rb = (int32_t)d->row_of_wire[net->in1[g]];
+            const int32_t rc2 = (int32_t)d->row_of_wire[net->in2[g]];
+            G.kind = kGateMux;
+            G.lane0 = (int32_t)ld.size();
+            ld.push_back(LaneDesc{ra, rb, 1, 1, 0u - kMu, 0u, 0u, 0u});      // AND(a, b)
+            G.lane1 = (int32_t)ld.size();
+            ld.push_back(LaneDesc{ra, rc2, -1, 1, 0u - kMu, 0u, 0u, 0u});    // ANDNY(a, c)
+        } else {
+            uint32_t C; int32_t wa, wb;
+            gate_linear(t, &C, &wa, &wb);
+            const int32_t rb = (int32_t)d->row_of_wire[net->in1[g]];
+            G.kind = kGateBoot;
+            G.lane0 = (int32_t)ld.size();
+            ld.push_back(LaneDesc{ra, rb, wa, wb, C, 0u, 0u, 0u});
+        }
+        gd[k] = G;
+        d->lane_off[k + 1] = (int64_t)ld.size();
+        d->boot_prefix[k + 1] = d->boot_prefix[k] + (t == TB_NOT ? 0 : 1);
+    }
+    cudaError_t e = cudaSetDevice(c->device);
+    if (e == cudaSuccess && ng > 0) e = cudaMalloc(&d->gdesc, gd.size() * sizeof(GateDesc));
+    if (e == cudaSuccess && !ld.empty()) e = cudaMalloc(&d->ldesc, ld.size() * sizeof(LaneDesc));
+    if (e == cudaSuccess && ng > 0) e = cudaMemcpy(d->gdesc, gd.data(), gd.size() * sizeof(GateDesc), cudaMemcpyHostToDevice);
+    if (e == cudaSuccess && !ld.empty()) e = cudaMemcpy(d->ldesc, ld.data(), ld.size() * sizeof(LaneDesc), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+        tb_netlist_free(c, d);
+        return cuda_fail(e, "tb_netlist_upload");
+    }
+    *out = d;
+    return TB_OK;
+}
+
+extern "C" int tb_netlist_free(tb_ctx* c, tb_dev_netlist* d) {
+    if (!d) return TB_OK;
+    if (c) cudaSetDevice(c->device);
+    cudaFree(d->gdesc);
+    cudaFree(d->ldesc);
+    delete d;
+    return TB_OK;
+}
+
+extern "C" int tb_netlist_info(const tb_dev_netlist* d, int64_t* n_levels, int64_t* n_rows) {
+    if (!d) return fail(TB_EINVAL, "null netlist");
+    if (n_levels) *n_levels = d->n_levels;
+    if (n_rows) *n_rows = d->n_inputs + d->n_gates;
+    return TB_OK;
+}
+
+extern "C" int tb_netlist_wire_rows(const tb_dev_netlist* d, int64_t* row_of_wire) {
+    if (!d || !row_of_wire) return fail(TB_EINVAL, "null argument");
+    std::copy(d->row_of_wire.begin(), d->row_of_wire.end(), row_of_wire);
+    return TB_OK;
+}
+
+extern "C" int tb_netlist_level(const tb_dev_netlist* d, int64_t level, int64_t* row0, int64_t* n_gates,
+                                int64_t* n_boot, int64_t* n_lanes) {
+    if (!d) return fail(TB_EINVAL, "null netlist");
+    if (level < 1 || level > d->n_levels) return fail(TB_EINVAL, "level out of range");
+    const int64_t a = d->level_off[level - 1], b = d->level_off[level];
+    if (row0) *row0 = d->n_inputs + a;
+    if (n_gates) *n_gates = b - a;
+    if (n_boot) *n_boot = d->boot_prefix[b] - d->boot_prefix[a];
+    if (n_lanes) *n_lanes = d->lane_off[b] - d->lane_off[a];
+    return TB_OK;
+}
+
+extern "C" int tb_run_level(tb_ctx* c, const tb_dev_netlist* d, int64_t level, int64_t g0, int64_t g1,
+                            uint32_t* wires, int64_t stride, tb_stream stream) {
+    int rc = check_ready(c);
+    if (rc) return rc;
+    if (!d || !wires) return fail(TB_EINVAL, "null argument");
+    if (stride < kn + 1) return fail(TB_EINVAL, "stride < n + 1");
+    if (level < 1 || level > d->n_levels) return fail(TB_EINVAL, "level out of range");
+    const int64_t a = d->level_off[level - 1], b = d->level_off[level];
+    if (g0 < 0 || g1 < g0 || a + g1 > b) return fail(TB_EINVAL, "gate range outside the level");
+    if (g0 == g1) return TB_OK;
+    TB_CUDA(cudaSetDevice(c->device));
+    const int64_t G0 = a + g0, G1 = a + g1;
+    const int64_t l0 = d->lane_off[G0], l1 = d->lane_off[G1];
+    if ((rc = grow_lanes(c, std::max<int64_t>(l1 - l0, 1)))) return rc;
+    cudaStream_t st = (cudaStream_t)stream;
+    if ((rc = run_br(c, wires, wires, wires, stride, d->ldesc + l0, l1 - l0, c->lanebuf, kLaneStride, st))) return rc;
+    return run_ks(c, c->lanebuf, l0, kLaneStride, d->gdesc + G0, G1 - G0, wires, stride, wires, stride, st);
+}
+
+extern "C" int tb_run_netlist(tb_ctx* c, const tb_dev_netlist* d, uint32_t* wires, int64_t stride, tb_stream stream) {
+    if (!d) return fail(TB_EINVAL, "null netlist");
+    for (int64_t L = 1; L <= d->n_levels; L++) {
+        const int64_t n = d->level_off[L] - d->level_off[L - 1];
+        int rc = tb_run_level(c, d, L, 0, n, wires, stride, stream);
+        if (rc) return rc;
+    }
+    return TB_OK;
+}

@@ -1,0 +1,45 @@
+"""Multi-GPU level loop.
+
+The paper's backend runs Algorithm 1 and submits every gate of `C - finished` as an independent job
+(P:198-203); its only communication is shipping 2.46 KB ciphertexts.  On one 8xB200 box
+the same structure becomes: every rank holds the keys (P:239's broadcast, done once at load) and the whole wire
+array; each level's gates are split into R contiguous chunks, rank r evaluates chunk r, and one in-place
+all-gather over NCCL/NVLink completes the level's output rows on every rank before the next level starts.
+Output bytes are independent of R (integer-exact kernels), so the result is byte-identical for R = 1..8.
+"""
+from __future__ import annotations
+
+
+def shard(n_gates: int, world: int, rank: int):
+    """(g0, g1, chunk): rank's contiguous gate range of a level and the padded chunk size."""
+    chunk = -(-n_gates // world) if n_gates else 0
+    g0 = min(rank * chunk, n_gates)
+    g1 = min((rank + 1) * chunk, n_gates)
+    return g0, g1, chunk
+
+
+def slack_rows(levels, n_rows: int, world: int) -> int:
+    """Rows past n_rows that the padded all-gather of some level may touch."""
+    need = 0
+    for row0, ng in levels:
+        _, _, chunk = shard(ng, world, 0)
+        need = max(need, row0 + world * chunk - n_rows)
+    return need
+
+
+def level_loop(levels, wires, run_level, group=None):
+    """levels: [(row0, n_gates)] for levels 1..L; run_level(level, g0, g1) evaluates a gate range of a level
+    into `wires` (a [rows, stride] tensor); with a process group of R > 1 ranks the level's output rows are
+    all-gathered in place after each level."""
+    import torch.distributed as dist
+    R = dist.get_world_size(group) if group is not None else 1
+    r = dist.get_rank(group) if group is not None else 0
+    for L, (row0, ng) in enumerate(levels, start=1):
+        g0, g1, chunk = shard(ng, R, r)
+        if R > 1 and row0 + R * chunk > wires.shape[0]:
+            raise ValueError("wire array needs slack rows for the padded all-gather (see slack_rows)")
+        if g1 > g0:
+            run_level(L, g0, g1)
+        if R > 1 and chunk:
+            dist.all_gather_into_tensor(wires[row0:row0 + R * chunk], wires[row0 + r * chunk:row0 + (r + 1) * chunk],
+                                        group=group)
