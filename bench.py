@@ -1,0 +1,319 @@
+#!/usr/bin/env python
+"""bench.py -- bootstrapped gates/s of the B200 TFHE hot path (BASELINE.json metric), one JSON line.
+
+Workload (BASELINE configs[2], the throughput sweep): one Algorithm-1 level of
+G independent NAND/XOR gates per GPU (seeded 50/50 mix, two fresh input ciphertexts per gate), tfhe-lib
+128-bit parameters.  A step = the whole hot path over that level: linear combination, mod switch, 630 CMux
+blind rotation, extraction, key switch, and for N > 1 the in-place NCCL all-gather of the
+level's output rows.  Weak scaling: G gates per GPU, N*G in total.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--gates-per-gpu G] [--impl ours|reference]
+
+`value` = N*G*K / (max over ranks of the CUDA-event time of the K steps).  `e2e` = the same metric through the
+C ABI with HOST buffers (tb_run_netlist_host: pinned inputs H2D, all levels, outputs D2H, synchronise) per
+step.  `cpu_baseline` = the CPU oracle (oracle/, schoolbook TFHE) timed on this host's cores on a bounded
+sample of the same workload.  --impl reference times that oracle alone as the reference arm.
+Key material and ciphertexts in the timed GPU arm are seeded uniform words: TFHE evaluation is
+data-oblivious, so timing does not depend on them; bit-exactness on this exact configuration is
+checked by tests/test_gpu_parity.py::test_throughput_level_bench_size_sampled.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "bootstrapped gates/sec (box, device-timed) at 1/2/4/8 B200; % of roofline"
+UNIT = "gates/s"
+CMUX_BFLY = 12 * 5 * 1024          # 12 negacyclic NTTs of N = 1024 per CMux step (6 forward + 6 inverse)
+CMUX_MAC = 6 * 6 * 1024            # pointwise 64-bit multiply-accumulates per CMux step
+N_LWE = 630
+
+
+def workload_name(G):
+    return ("cfg3 throughput sweep: one level of %d independent NAND/XOR gates per GPU (seeded 50/50), "
+            "tfhe-lib 128-bit params n=630 N=1024 k=1 l=3 Bgbit=7 KS t=8 base 4" % G)
+
+
+# ------------------------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi sampled every 200 ms while the timed region runs (B200_PROFILING.md clocks line)."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_id: str):
+        self.gpu_id, self.rows, self.proc = gpu_id, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", self.gpu_id, "--query-gpu=" + self.Q,
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm = [float(r[0]) for r in self.rows if len(r) >= 7 and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) >= 7 and r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in self.rows if len(r) >= 7 for k in range(4) if r[3 + k] == "Active"})
+        pw = [float(r[2]) for r in self.rows if len(r) >= 7 and r[2].replace(".", "").isdigit()]
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(sm), "power_w_max": max(pw) if pw else None}
+
+
+def gpu_id_for(dev: int) -> str:
+    import torch
+    try:
+        u = str(torch.cuda.get_device_properties(dev).uuid)
+        return u if u.startswith("GPU-") else "GPU-" + u
+    except Exception:
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+        return vis.split(",")[dev] if vis else str(dev)
+
+
+# ------------------------------------------------------------------------------------------------ oracle
+def oracle_rate(G_types, seconds_hint=None):
+    """Time the CPU oracle on a bounded sample of the workload: 4 gates per host thread (NAND/XOR as in
+    the GPU arm) with real seeded keys; returns (gates/s, threads, sample description)."""
+    import numpy as np
+    import oracle as O
+    import synth
+    threads = O.max_threads()
+    keys = O.keygen(O.DEFAULT, seed=99)
+    ns = 4 * threads
+    types = np.asarray(G_types[:ns], np.int32)
+    bits = synth.random_bits(2 * ns, 98)
+    ca, cb = O.encrypt_bits(keys, bits[0::2], 1), O.encrypt_bits(keys, bits[1::2], 2)
+    t0 = time.perf_counter()
+    O.gates(keys, types, ca, cb, nthreads=threads)
+    dt = time.perf_counter() - t0
+    return ns / dt, threads, "%d NAND/XOR gates of the same workload (4 per thread) on %d host threads, %.1f s" % (
+        ns, threads, dt)
+
+
+def run_reference(args, rank):
+    """--impl reference: the CPU oracle as it stands, on this host's cores (rank 0 only)."""
+    if rank != 0:
+        return
+    import numpy as np
+    import oracle as O
+    import synth
+    O.build()
+    threads = O.max_threads()
+    keys = O.keygen(O.DEFAULT, seed=99)
+    n = synth.independent_level(threads * (args.warmup + args.steps), seed=1)
+    bits = synth.random_bits(2 * n["type"].size, 2)
+    ca, cb = O.encrypt_bits(keys, bits[0::2], 3), O.encrypt_bits(keys, bits[1::2], 4)
+    per = threads                     # one gate per thread per step: a bounded sample of the workload
+    times = []
+    for s in range(args.warmup + args.steps):
+        sl = slice(s * per, (s + 1) * per)
+        t0 = time.perf_counter()
+        O.gates(keys, n["type"][sl], ca[sl], cb[sl], nthreads=threads)
+        times.append(time.perf_counter() - t0)
+    t = sum(times[args.warmup:])
+    value = per * args.steps / t
+    sample = "%d steps x %d NAND/XOR gates (one per host thread) of the cfg3 workload" % (args.steps, per)
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic (seeded keys and inputs)",
+        "config": {"workload": workload_name(args.gates_per_gpu), "oracle": "plain C schoolbook TFHE (oracle/)"},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+# ------------------------------------------------------------------------------------------------ ours
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--gates-per-gpu", type=int, default=65536)
+    ap.add_argument("--lanes-per-cta", type=int, default=2)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank)
+        return
+    if args.warmup < 3:
+        args.warmup = 3                                  # timing rule: >= 3 warm-up steps
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ispass_maxw23_b200 as tb
+    import synth
+
+    torch.cuda.set_device(local)
+    group = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        group = dist.group.WORLD
+    G = args.gates_per_gpu
+    total = G * world
+    ctx = tb.Context(local)
+    ctx.set_lanes_per_cta(args.lanes_per_cta)
+    ctx.load_keys(synth.random_words(tb.BK_WORDS, 11), synth.random_words(tb.KSK_WORDS, 12))
+    n = synth.independent_level(total, seed=13)
+    net = tb.Netlist(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"], outputs=n["outputs"])
+    dnet = ctx.upload(net)
+    wires = ctx.wire_array(dnet, tb.slack_rows(dnet, world))
+    gen = torch.Generator(device=ctx.device)
+    gen.manual_seed(14)
+    wires[:n["n_inputs"]].random_(-2 ** 31, 2 ** 31 - 1, generator=gen)     # resident inputs (> L2)
+
+    def step():
+        ctx.run_netlist(dnet, wires, group)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(gpu_id_for(local))
+    sampler.start()
+    time.sleep(0.3)
+    if group is not None:
+        dist.barrier()
+    torch.cuda.synchronize()
+    ctx.profile(True)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record()
+    for _ in range(args.steps):
+        step()
+    ev1.record()
+    torch.cuda.synchronize()
+    if group is not None:
+        dist.barrier()
+    clocks = sampler.stop()
+    ms = ev0.elapsed_time(ev1)
+    br_ms, br_n, ks_ms, ks_n = ctx.profile_read()
+    ctx.profile(False)
+    if group is not None:
+        t = torch.tensor([ms], device=ctx.device)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    value = total * args.steps / (ms / 1e3)
+
+    # roofline of the dominant kernel (br_kernel): integer butterflies + MACs vs the microbenchmarked rate
+    bfly_rate, mac_rate = ctx.microbench()
+    g0, g1, _ = tb.parallel.shard(total, world, rank)
+    lanes_per_launch = g1 - g0
+    work = N_LWE * (CMUX_BFLY + CMUX_MAC * bfly_rate / mac_rate) * lanes_per_launch   # butterfly-equivalents
+    br_launch_s = br_ms / max(br_n, 1) / 1e3
+    achieved = work / br_launch_s
+    traffic = None
+    prof_path = os.path.join(ROOT, "profiles", "ncu_br_kernel_summary.json")
+    if os.path.exists(prof_path):
+        try:
+            pj = json.load(open(prof_path))
+            if pj.get("lanes") == lanes_per_launch and pj.get("lanes_per_cta") == args.lanes_per_cta:
+                traffic = pj.get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    roofline = {"bound": "alu", "achieved": achieved / 1e9, "peak": bfly_rate / 1e9, "unit": "Gbutterfly-eq/s",
+                "frac": achieved / bfly_rate, "traffic": traffic,
+                "kernel": "br_kernel", "kernel_ms_per_launch": br_launch_s * 1e3,
+                "kernel_share_of_step": br_ms / ms if ms else None,
+                "ks_kernel_ms_per_launch": ks_ms / max(ks_n, 1),
+                "peak_source": "tb_microbench on this GPU in this run: the kernels' own lazy Shoup butterfly, "
+                               "register resident, all SMs (%.3g bfly/s; 64-bit MAC %.3g/s)" % (bfly_rate, mac_rate),
+                "work_per_bootstrap": "630 x (61,440 butterflies + 36,864 MAC x bfly_rate/mac_rate)"}
+
+    # narrow-level latency (one gate)
+    lat = None
+    one = ctx.empty(2)
+    one.random_(-2 ** 31, 2 ** 31 - 1, generator=gen)
+    outl = ctx.empty(1)
+    for _ in range(2):
+        ctx.gates(tb.NAND, one[:1], one[1:2], out=outl)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(3):
+        ctx.gates(tb.NAND, one[:1], one[1:2], out=outl)
+    e1.record()
+    torch.cuda.synchronize()
+    lat = e0.elapsed_time(e1) / 3
+
+    # e2e through the C ABI with host buffers (per-rank replica of the per-GPU workload)
+    e2e = None
+    if not args.no_e2e:
+        nr = synth.independent_level(G, seed=15)
+        rnet = ctx.upload(tb.Netlist(nr["n_inputs"], nr["type"], nr["in0"], nr["in1"], nr["in2"]))
+        hin = torch.empty((nr["n_inputs"], tb.CT_WORDS), dtype=torch.int32, pin_memory=True)
+        hin.random_(-2 ** 31, 2 ** 31 - 1)
+        hout = torch.empty((G, tb.CT_WORDS), dtype=torch.int32, pin_memory=True)
+        ow = np.ascontiguousarray(nr["outputs"], np.int64)
+        ctx.run_netlist_host_into(rnet, hin, ow, hout)
+        if group is not None:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            ctx.run_netlist_host_into(rnet, hin, ow, hout)
+        dt = time.perf_counter() - t0
+        if group is not None:
+            t = torch.tensor([dt], device=ctx.device, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            dt = float(t.item())
+        e2e = {"value": G * world * args.steps / dt, "unit": UNIT,
+               "h2d_bytes_per_step": int(nr["n_inputs"] * tb.CT_WORDS * 4),
+               "d2h_bytes_per_step": int(G * tb.CT_WORDS * 4),
+               "api": "tb_run_netlist_host (pinned host inputs -> device, run, outputs -> host, per rank)"}
+        rnet.free()
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, cores, sample = oracle_rate(n["type"])
+        cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
+
+    if rank == 0:
+        print(json.dumps({
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic: seeded uniform key material and ciphertexts (evaluation is data-oblivious, P:160)",
+            "config": {"workload": workload_name(G), "gates_per_gpu": G, "total_gates": total,
+                       "parallelism": "dp%d (level sharded, NCCL all-gather of output rows)" % world,
+                       "lanes_per_cta": args.lanes_per_cta,
+                       "l2": "inputs larger than L2 (%.0f MB of input ciphertexts per GPU)" % (2 * G * 2524 / 1e6)},
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+            "gpu_launches": br_n + ks_n,
+            "latency_ms": {"level_of_%d_gates" % total: ms / args.steps, "level_of_1_gate": lat},
+        }), flush=True)
+    if group is not None:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

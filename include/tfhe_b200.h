@@ -124,6 +124,20 @@ int tb_run_level(tb_ctx* ctx, const tb_dev_netlist* dnet, int64_t level, int64_t
 /* All levels in order on one device (single-GPU path).  Async. */
 int tb_run_netlist(tb_ctx* ctx, const tb_dev_netlist* dnet, uint32_t* wires, int64_t stride, tb_stream stream);
 
+/* End-to-end netlist evaluation through HOST buffers: copies the n_inputs input ciphertexts (rows of
+ * in_stride words, host) into a context-owned device wire array, runs every level, gathers the rows of
+ * the n_outputs wires listed in output_wires (original wire ids, host array) and copies them to
+ * host_outputs (rows of out_stride >= 631 words).  Synchronous. */
+int tb_run_netlist_host(tb_ctx* ctx, const tb_dev_netlist* dnet, const uint32_t* host_inputs, int64_t in_stride,
+                        const int64_t* output_wires, int64_t n_outputs, uint32_t* host_outputs, int64_t out_stride);
+
+/* ---- per-kernel timing (CUDA events recorded around every launch on the launching stream) ---------- */
+/* enable != 0 starts recording (and clears previous records); 0 stops. */
+int tb_profile_enable(tb_ctx* ctx, int enable);
+/* Synchronises the recorded events and returns the summed device time (ms) and launch counts of the
+ * blind-rotation kernel and of the key-switch kernel since tb_profile_enable(ctx, 1). */
+int tb_profile_read(tb_ctx* ctx, double* br_ms, int64_t* br_launches, double* ks_ms, int64_t* ks_launches);
+
 /* ---- diagnostics used by the parity tests ---------------------------------------------------------- */
 /* Blind rotation + extraction only: out[g] (N+1 words, rows `out_stride` apart) = Extract(BlindRotate(
  * ModSwitch(in[g]))) with test vector mu = 1/8 -- SURVEY 8(a) a2-a5 without the key switch.  Async. */

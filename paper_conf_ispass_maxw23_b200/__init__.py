@@ -213,6 +213,36 @@ class Context:
         parallel.level_loop([(row0, ng) for row0, ng, _, _ in dnet.levels], wires,
                             lambda L, g0, g1: self.run_level(dnet, L, g0, g1, wires, stream), group)
 
+    def run_netlist_host(self, dnet: DevNetlist, inputs: np.ndarray, output_wires) -> np.ndarray:
+        """End-to-end through HOST buffers (tb_run_netlist_host): input ciphertexts [n_inputs, >=631] u32 ->
+        output ciphertexts [len(output_wires), 631] u32.  Pinned host memory makes the copies faster."""
+        inputs = np.ascontiguousarray(inputs, np.uint32) if not isinstance(inputs, np.ndarray) or \
+            inputs.dtype != np.uint32 or not inputs.flags.c_contiguous else inputs
+        ow = np.ascontiguousarray(output_wires, np.int64)
+        out = np.empty((ow.size, CT_WORDS), np.uint32)
+        _native.check(_native.lib().tb_run_netlist_host(self._h, dnet._h, inputs.ctypes.data, inputs.shape[1],
+                                                        ow.ctypes.data, ow.size, out.ctypes.data, CT_WORDS))
+        return out
+
+    def run_netlist_host_into(self, dnet: DevNetlist, inputs: torch.Tensor, output_wires: np.ndarray,
+                              out: torch.Tensor) -> None:
+        """Same with caller-owned (pinned) host tensors: inputs [n_inputs, stride] int32, out [n, stride]."""
+        _native.check(_native.lib().tb_run_netlist_host(self._h, dnet._h, ctypes.c_void_p(inputs.data_ptr()),
+                                                        inputs.stride(0), output_wires.ctypes.data,
+                                                        output_wires.size, ctypes.c_void_p(out.data_ptr()),
+                                                        out.stride(0)))
+
+    # ---- per-kernel device time (CUDA events around each launch) ----
+    def profile(self, enable: bool):
+        _native.check(_native.lib().tb_profile_enable(self._h, 1 if enable else 0))
+
+    def profile_read(self):
+        """-> (br_ms, br_launches, ks_ms, ks_launches) since profile(True)."""
+        a, b, c, d = ctypes.c_double(), ctypes.c_int64(), ctypes.c_double(), ctypes.c_int64()
+        _native.check(_native.lib().tb_profile_read(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c),
+                                                    ctypes.byref(d)))
+        return a.value, int(b.value), c.value, int(d.value)
+
     def close(self):
         if getattr(self, "_h", None):
             _native.lib().tb_ctx_destroy(self._h)

@@ -78,6 +78,10 @@ SIGNATURES = {
     "tb_netlist_level": (ctypes.c_int, [_vp, _i64, _pi64, _pi64, _pi64, _pi64]),
     "tb_run_level": (ctypes.c_int, [_vp, _vp, _i64, _i64, _i64, _vp, _i64, _vp]),
     "tb_run_netlist": (ctypes.c_int, [_vp, _vp, _vp, _i64, _vp]),
+    "tb_run_netlist_host": (ctypes.c_int, [_vp, _vp, _vp, _i64, _vp, _i64, _vp, _i64]),
+    "tb_profile_enable": (ctypes.c_int, [_vp, ctypes.c_int]),
+    "tb_profile_read": (ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), _pi64, ctypes.POINTER(ctypes.c_double),
+                                       _pi64]),
     "tb_bootstrap_wo_ks": (ctypes.c_int, [_vp, _vp, _i64, _vp, _i64, _i64, _vp]),
     "tb_keyswitch": (ctypes.c_int, [_vp, _vp, _i64, _vp, _i64, _i64, _vp]),
     "tb_ntt_muladd6": (ctypes.c_int, [_vp, _vp, _vp, _vp]),

@@ -36,6 +36,7 @@ struct KsArgs {
 };
 
 int launch_br(const BrArgs& A, int G, cudaStream_t st);
+int launch_br6(const BrArgs& A, int G, cudaStream_t st);
 size_t br_smem_bytes(int G);
 void launch_bk_to_ntt(const uint32_t* bk, uint32_t* bkhat, const uint2* twF, uint32_t ninv, uint32_t ninvp,
                       cudaStream_t st);
@@ -49,4 +50,9 @@ int launch_ntt_muladd6(const int32_t* digits, const uint32_t* polys, uint32_t* r
                        const uint2* twI, uint32_t ninv, uint32_t ninvp, cudaStream_t st);
 int run_microbench(int iters, double* bfly, double* mac);
 
+}  // namespace tb
+
+namespace tb {
+void launch_gather_rows(const uint32_t* src, int64_t stride, const int64_t* rows, int64_t n, uint32_t* out,
+                        cudaStream_t st);
 }  // namespace tb

@@ -6,6 +6,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -58,6 +59,7 @@ static uint32_t brv10(uint32_t k) {
 struct tb_ctx {
     int device = 0;
     int lanes_per_cta = 2;
+    int variant = 6;                        // blind-rotation kernel: 6 = br6_kernel (6 warps/lane), 2 = br_kernel
     cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
     uint2* twF = nullptr;                   // [31][32]
     uint2* twI = nullptr;
@@ -73,7 +75,38 @@ struct tb_ctx {
     int64_t desc_rows = 0;
     uint32_t* stage = nullptr;              // tb_gates_host staging
     size_t stage_words = 0;
+    uint32_t* hwires = nullptr;             // tb_run_netlist_host device wire array
+    size_t hwires_words = 0;
+    int64_t* hidx = nullptr;                // tb_run_netlist_host gather rows
+    int64_t hidx_n = 0;
+    // per-kernel event timing (tb_profile_*)
+    bool prof = false;
+    std::vector<cudaEvent_t> ev_pool;
+    size_t ev_used = 0;
+    std::vector<std::pair<int, size_t>> ev_rec;   // (kind 0 = br / 1 = ks, index of start event)
 };
+
+static cudaEvent_t next_event(tb_ctx* c) {
+    if (c->ev_used == c->ev_pool.size()) {
+        cudaEvent_t e;
+        if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+        c->ev_pool.push_back(e);
+    }
+    return c->ev_pool[c->ev_used++];
+}
+// record a start event before a launch of `kind`; returns the record slot or -1
+static long prof_begin(tb_ctx* c, int kind, cudaStream_t st) {
+    if (!c->prof) return -1;
+    cudaEvent_t a = next_event(c), b = next_event(c);
+    if (!a || !b) return -1;
+    cudaEventRecord(a, st);
+    c->ev_rec.push_back({kind, c->ev_used - 2});
+    return (long)c->ev_rec.size() - 1;
+}
+static void prof_end(tb_ctx* c, long slot, cudaStream_t st) {
+    if (slot < 0) return;
+    cudaEventRecord(c->ev_pool[c->ev_rec[slot].second + 1], st);
+}
 
 struct tb_dev_netlist {
     int64_t n_inputs = 0, n_gates = 0, n_levels = 0;
@@ -137,6 +170,7 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
     tb_ctx* c = new (std::nothrow) tb_ctx();
     if (!c) return fail(TB_ENOMEM, "host allocation failed");
     c->device = dev;
+    if (const char* v = getenv("TB_BR_VARIANT")) c->variant = atoi(v);   // experiment knob (6 or 2)
 
     // psi: primitive 2N-th root of unity mod p (psi^N = -1)
     uint32_t psi = 0;
@@ -192,6 +226,9 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
     cudaFree(c->ldesc);
     cudaFree(c->gdesc);
     cudaFree(c->stage);
+    cudaFree(c->hwires);
+    cudaFree(c->hidx);
+    for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
     if (c->own) cudaStreamDestroy(c->own);
     delete c;
     return TB_OK;
@@ -286,7 +323,9 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     A.src0 = s0; A.src1 = s1; A.src2 = s2; A.src_stride = sstride;
     A.lanes = lanes; A.nlanes = (int32_t)nlanes; A.bkhat = c->bkhat; A.twF = c->twF; A.twI = c->twI;
     A.out = out; A.out_stride = ostride;
-    int rc = launch_br(A, c->lanes_per_cta, st);
+    const long slot = prof_begin(c, 0, st);
+    int rc = c->variant == 6 ? launch_br6(A, c->lanes_per_cta, st) : launch_br(A, c->lanes_per_cta, st);
+    prof_end(c, slot, st);
     if (rc) return fail(TB_ECUDA, "blind-rotation kernel attribute/launch failed");
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "br_kernel launch");
@@ -300,7 +339,9 @@ static int run_ks(tb_ctx* c, const uint32_t* lanes, int64_t lane_base, int64_t l
     A.lanes = lanes; A.lane_base = (int32_t)lane_base; A.lane_stride = lane_stride; A.gates = gates;
     A.ngates = (int32_t)ngates; A.ksk = c->ksk; A.out = out; A.out_stride = ostride; A.not_src = not_src;
     A.not_stride = not_stride;
+    const long slot = prof_begin(c, 1, st);
     launch_ks(A, st);
+    prof_end(c, slot, st);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "ks_kernel launch");
     return TB_OK;
@@ -618,5 +659,95 @@ extern "C" int tb_run_netlist(tb_ctx* c, const tb_dev_netlist* d, uint32_t* wire
         int rc = tb_run_level(c, d, L, 0, n, wires, stride, stream);
         if (rc) return rc;
     }
+    return TB_OK;
+}
+
+// ------------------------------------------------------------------------------------------ profiling
+extern "C" int tb_profile_enable(tb_ctx* c, int enable) {
+    if (!c) return fail(TB_EINVAL, "null context");
+    TB_CUDA(cudaSetDevice(c->device));
+    if (enable) {
+        c->ev_used = 0;
+        c->ev_rec.clear();
+    }
+    c->prof = enable != 0;
+    return TB_OK;
+}
+
+extern "C" int tb_profile_read(tb_ctx* c, double* br_ms, int64_t* br_n, double* ks_ms, int64_t* ks_n) {
+    if (!c) return fail(TB_EINVAL, "null context");
+    TB_CUDA(cudaSetDevice(c->device));
+    double t[2] = {0, 0};
+    int64_t n[2] = {0, 0};
+    for (const auto& r : c->ev_rec) {
+        TB_CUDA(cudaEventSynchronize(c->ev_pool[r.second + 1]));
+        float ms = 0;
+        TB_CUDA(cudaEventElapsedTime(&ms, c->ev_pool[r.second], c->ev_pool[r.second + 1]));
+        t[r.first] += ms;
+        n[r.first]++;
+    }
+    if (br_ms) *br_ms = t[0];
+    if (br_n) *br_n = n[0];
+    if (ks_ms) *ks_ms = t[1];
+    if (ks_n) *ks_n = n[1];
+    return TB_OK;
+}
+
+// ------------------------------------------------------------------------------------------ e2e host path
+extern "C" int tb_run_netlist_host(tb_ctx* c, const tb_dev_netlist* d, const uint32_t* hin, int64_t in_stride,
+                                   const int64_t* outw, int64_t n_out, uint32_t* hout, int64_t out_stride) {
+    int rc = check_ready(c);
+    if (rc) return rc;
+    if (!d || (d->n_inputs > 0 && !hin) || (n_out > 0 && (!outw || !hout))) return fail(TB_EINVAL, "null argument");
+    if (in_stride < kn + 1 || out_stride < kn + 1 || n_out < 0) return fail(TB_EINVAL, "bad stride or count");
+    const int64_t nw = d->n_inputs + d->n_gates;
+    std::vector<int64_t> rows((size_t)n_out);
+    bool contiguous = true;
+    for (int64_t k = 0; k < n_out; k++) {
+        if (outw[k] < 0 || outw[k] >= nw) return fail(TB_EINVAL, "output wire out of range");
+        rows[k] = d->row_of_wire[outw[k]];
+        if (k && rows[k] != rows[k - 1] + 1) contiguous = false;
+    }
+    TB_CUDA(cudaSetDevice(c->device));
+    const int64_t S = kKsRow;                        // 632-word device rows
+    const size_t words = (size_t)(nw + std::max<int64_t>(n_out, 1)) * S;
+    if (c->hwires_words < words) {
+        cudaFree(c->hwires);
+        c->hwires = nullptr;
+        c->hwires_words = 0;
+        if (cudaMalloc(&c->hwires, words * 4) != cudaSuccess) {
+            cudaGetLastError();
+            return fail(TB_ENOMEM, "wire array allocation failed");
+        }
+        c->hwires_words = words;
+    }
+    uint32_t* gather = c->hwires + (size_t)nw * S;
+    if (d->n_inputs > 0)
+        TB_CUDA(cudaMemcpy2DAsync(c->hwires, S * 4, hin, in_stride * 4, (kn + 1) * 4, d->n_inputs,
+                                  cudaMemcpyHostToDevice, c->own));
+    rc = tb_run_netlist(c, d, c->hwires, S, (tb_stream)c->own);
+    if (rc) return rc;
+    if (n_out > 0) {
+        const uint32_t* src = c->hwires + (size_t)rows[0] * S;
+        if (!contiguous) {
+            if (c->hidx_n < n_out) {
+                cudaFree(c->hidx);
+                c->hidx = nullptr;
+                c->hidx_n = 0;
+                if (cudaMalloc(&c->hidx, n_out * 8) != cudaSuccess) {
+                    cudaGetLastError();
+                    return fail(TB_ENOMEM, "index allocation failed");
+                }
+                c->hidx_n = n_out;
+            }
+            TB_CUDA(cudaMemcpyAsync(c->hidx, rows.data(), n_out * 8, cudaMemcpyHostToDevice, c->own));
+            launch_gather_rows(c->hwires, S, c->hidx, n_out, gather, c->own);
+            TB_CUDA(cudaGetLastError());
+            src = gather;
+        }
+        TB_CUDA(cudaMemcpy2DAsync(hout, out_stride * 4, src, S * 4, (kn + 1) * 4, n_out, cudaMemcpyDeviceToHost,
+                                  c->own));
+    }
+    TB_CUDA(cudaStreamSynchronize(c->own));
     return TB_OK;
 }
