@@ -225,13 +225,22 @@ def main():
         ms = float(t.item())
     value = total * args.steps / (ms / 1e3)
 
-    # roofline of the dominant kernel (br_kernel): integer butterflies + MACs vs the microbenchmarked rate
+    # roofline of the dominant kernel (blind rotation): the integer-multiply (FMA-heavy) pipe.  Algorithmic
+    # work = IMAD issue slots of the method's modular arithmetic: per CMux step
+    # 61,440 Shoup mulmods x 4 slots (IMAD + IMAD.HI(2) + IMAD) + 36,864 64-bit MACs x 2 (IMAD.WIDE) + 6,144
+    # MAC reductions x 5.  Peak = 148 SMs x 64 IMAD lanes/clk (fma pipe: 16 lanes/clk/SMSP, B300_MICROARCH
+    # "Pipe rates") x the median SM clock sampled during the timed region.
     bfly_rate, mac_rate = ctx.microbench()
     g0, g1, _ = tb.parallel.shard(total, world, rank)
     lanes_per_launch = g1 - g0
-    work = N_LWE * (CMUX_BFLY + CMUX_MAC * bfly_rate / mac_rate) * lanes_per_launch   # butterfly-equivalents
+    slots_per_bootstrap = N_LWE * (CMUX_BFLY * 4 + CMUX_MAC * 2 + 6 * 1024 * 5)
+    work = slots_per_bootstrap * lanes_per_launch
     br_launch_s = br_ms / max(br_n, 1) / 1e3
     achieved = work / br_launch_s
+    sm_count = torch.cuda.get_device_properties(local).multi_processor_count
+    clk_mhz = clocks.get("sm_mhz") or 1965.0
+    peak = sm_count * 64 * clk_mhz * 1e6
+    bfly_work = N_LWE * (CMUX_BFLY + CMUX_MAC * bfly_rate / mac_rate) * lanes_per_launch
     traffic = None
     prof_path = os.path.join(ROOT, "profiles", "ncu_br_kernel_summary.json")
     if os.path.exists(prof_path):
@@ -241,14 +250,18 @@ def main():
                 traffic = pj.get("dram_bytes_per_launch")
         except Exception:
             traffic = None
-    roofline = {"bound": "alu", "achieved": achieved / 1e9, "peak": bfly_rate / 1e9, "unit": "Gbutterfly-eq/s",
-                "frac": achieved / bfly_rate, "traffic": traffic,
-                "kernel": "br_kernel", "kernel_ms_per_launch": br_launch_s * 1e3,
+    roofline = {"bound": "alu", "achieved": achieved / 1e9, "peak": peak / 1e9, "unit": "G IMAD-slots/s",
+                "frac": achieved / peak, "traffic": traffic,
+                "kernel": "br6_kernel (blind rotation + extraction)", "kernel_ms_per_launch": br_launch_s * 1e3,
                 "kernel_share_of_step": br_ms / ms if ms else None,
                 "ks_kernel_ms_per_launch": ks_ms / max(ks_n, 1),
-                "peak_source": "tb_microbench on this GPU in this run: the kernels' own lazy Shoup butterfly, "
-                               "register resident, all SMs (%.3g bfly/s; 64-bit MAC %.3g/s)" % (bfly_rate, mac_rate),
-                "work_per_bootstrap": "630 x (61,440 butterflies + 36,864 MAC x bfly_rate/mac_rate)"}
+                "peak_source": "derived: %d SMs x 64 IMAD lanes/clk x %.0f MHz (median SM clock in the timed region)"
+                               % (sm_count, clk_mhz),
+                "work_per_bootstrap": "%d IMAD slots = 630 x (61,440 mulmod x 4 + 36,864 MAC x 2 + 6,144 reductions x 5)"
+                                      % slots_per_bootstrap,
+                "bootstraps_per_s_at_peak": peak / slots_per_bootstrap,
+                "microbench_crosscheck": {"butterflies_per_s": bfly_rate, "macs_per_s": mac_rate,
+                                          "frac_of_microbench": bfly_work / br_launch_s / bfly_rate}}
 
     # narrow-level latency (one gate)
     lat = None

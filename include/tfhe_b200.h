@@ -102,6 +102,13 @@ typedef struct {
  * iteration of the while loop in which g first enters C - finished.  Writes *n_levels. */
 int tb_levelise(const tb_netlist* net, int64_t* level_of_gate, int64_t* n_levels);
 
+/* Host-only execution plan (no device needed): *n_levels; level_off[L] for L = 0..n_levels = offset of the
+ * first gate of level L+1 in level-sorted order (level_off[n_levels] = n_gates); row_of_wire[w] = the wire
+ * array row of wire w (inputs first, then level 1's outputs, level 2's, ...; ascending gate index inside a
+ * level).  Pass level_off = row_of_wire = NULL to query n_levels first.  This is the layout
+ * tb_netlist_upload uses and the one the multi-GPU level loop shards (contiguous output rows per level). */
+int tb_netlist_plan(const tb_netlist* net, int64_t* n_levels, int64_t* level_off, int64_t* row_of_wire);
+
 typedef struct tb_dev_netlist tb_dev_netlist;   /* library-owned device copy of a levelised netlist */
 
 /* Levelise, renumber wires so that every level's outputs form one contiguous block of rows (inputs first,

@@ -71,7 +71,8 @@ SIGNATURES = {
     "tb_gates": (ctypes.c_int, [_vp, ctypes.c_int, _vp, _vp, _vp, _vp, _i64, _i64, _vp]),
     "tb_gates_host": (ctypes.c_int, [_vp, ctypes.c_int, _vp, _vp, _vp, _vp, _i64, _i64]),
     "tb_levelise": (ctypes.c_int, [ctypes.POINTER(Netlist), _vp, _pi64]),
-    "tb_netlist_upload": (ctypes.c_int, [_vp, ctypes.POINTER(Netlist), ctypes.POINTER(_vp)]),
+    "tb_netlist_plan": (ctypes.c_int, [ctypes.POINTER(Netlist), _pi64, _vp, _vp]),
+    "tb_netlist_upload":(ctypes.c_int, [_vp, ctypes.POINTER(Netlist), ctypes.POINTER(_vp)]),
     "tb_netlist_free": (ctypes.c_int, [_vp, _vp]),
     "tb_netlist_info": (ctypes.c_int, [_vp, _pi64, _pi64]),
     "tb_netlist_wire_rows": (ctypes.c_int, [_vp, _vp]),

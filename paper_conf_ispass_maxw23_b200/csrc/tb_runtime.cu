@@ -521,35 +521,54 @@ extern "C" int tb_levelise(const tb_netlist* net, int64_t* level_of_gate, int64_
     return TB_OK;
 }
 
-extern "C" int tb_netlist_upload(tb_ctx* c, const tb_netlist* net, tb_dev_netlist** out) {
-    if (!c || !net || !out) return fail(TB_EINVAL, "null argument");
-    *out = nullptr;
+// Levelise (Algorithm 1) and renumber: inputs keep rows [0, n_inputs); the gates of level L follow those of
+// level L-1, ascending original index inside a level.  level_off (0-based, n_levels + 1 entries) are gate
+// offsets into that order; order[k] = original gate index of the k-th gate.
+static int plan_impl(const tb_netlist* net, int64_t* n_levels, std::vector<int64_t>& level_off,
+                     std::vector<int64_t>& order, std::vector<int64_t>& row_of_wire) {
     std::vector<int64_t> lv;
     int64_t nlev = 0;
     int rc = levelise_impl(net, lv, &nlev);
     if (rc) return rc;
     const int64_t ni = net->n_inputs, ng = net->n_gates;
-    if (ni + ng > INT32_MAX) return fail(TB_EINVAL, "netlist too large for 32-bit rows");
+    std::vector<int64_t> cnt((size_t)nlev + 2, 0);
+    for (int64_t g = 0; g < ng; g++) cnt[lv[g]]++;
+    level_off.assign((size_t)nlev + 1, 0);
+    for (int64_t L = 1; L <= nlev; L++) level_off[L] = level_off[L - 1] + cnt[L];
+    std::vector<int64_t> pos(level_off.begin(), level_off.end());
+    order.assign((size_t)ng, 0);
+    for (int64_t g = 0; g < ng; g++) order[pos[lv[g] - 1]++] = g;
+    row_of_wire.resize((size_t)(ni + ng));
+    for (int64_t w = 0; w < ni; w++) row_of_wire[w] = w;
+    for (int64_t k = 0; k < ng; k++) row_of_wire[ni + order[k]] = ni + k;
+    *n_levels = nlev;
+    return TB_OK;
+}
+
+extern "C" int tb_netlist_plan(const tb_netlist* net, int64_t* n_levels, int64_t* level_off, int64_t* row_of_wire) {
+    if (!net || !n_levels) return fail(TB_EINVAL, "null argument");
+    std::vector<int64_t> lo, order, rows;
+    int rc = plan_impl(net, n_levels, lo, order, rows);
+    if (rc) return rc;
+    if (level_off) std::copy(lo.begin(), lo.end(), level_off);
+    if (row_of_wire) std::copy(rows.begin(), rows.end(), row_of_wire);
+    return TB_OK;
+}
+
+extern "C" int tb_netlist_upload(tb_ctx* c, const tb_netlist* net, tb_dev_netlist** out) {
+    if (!c || !net || !out) return fail(TB_EINVAL, "null argument");
+    *out = nullptr;
+    if (net->n_inputs + net->n_gates > INT32_MAX) return fail(TB_EINVAL, "netlist too large for 32-bit rows");
     tb_dev_netlist* d = new (std::nothrow) tb_dev_netlist();
     if (!d) return fail(TB_ENOMEM, "host allocation failed");
-    d->n_inputs = ni; d->n_gates = ng; d->n_levels = nlev;
-    // counting sort by level (stable: ascending original index inside a level)
-    d->level_off.assign((size_t)nlev + 2, 0);
-    for (int64_t g = 0; g < ng; g++) d->level_off[lv[g]]++;
-    {
-        int64_t s = 0;
-        for (int64_t L = 1; L <= nlev; L++) { int64_t k = d->level_off[L]; d->level_off[L] = s; s += k; }
-        d->level_off[nlev + 1] = s;
+    std::vector<int64_t> order;
+    int rc = plan_impl(net, &d->n_levels, d->level_off, order, d->row_of_wire);
+    if (rc) {
+        delete d;
+        return rc;
     }
-    std::vector<int64_t> order((size_t)ng), pos(d->level_off.begin(), d->level_off.end());
-    for (int64_t g = 0; g < ng; g++) order[pos[lv[g]]++] = g;
-    // level_off[L] (1-based) -> store 0-based [n_levels + 1]
-    std::vector<int64_t> lo((size_t)nlev + 1);
-    for (int64_t L = 0; L <= nlev; L++) lo[L] = d->level_off[L + 1];
-    d->level_off.swap(lo);
-    d->row_of_wire.resize((size_t)(ni + ng));
-    for (int64_t w = 0; w < ni; w++) d->row_of_wire[w] = w;
-    for (int64_t k = 0; k < ng; k++) d->row_of_wire[ni + order[k]] = ni + k;
+    const int64_t ni = net->n_inputs, ng = net->n_gates;
+    d->n_inputs = ni; d->n_gates = ng;
     // descriptors in level-sorted order
     std::vector<GateDesc> gd((size_t)ng);
     std::vector<LaneDesc> ld;

@@ -63,6 +63,19 @@ class Netlist:
         _native.check(_native.lib().tb_levelise(ctypes.byref(s), lv.ctypes.data, ctypes.byref(nl)))
         return lv, int(nl.value)
 
+    def plan(self):
+        """Host-only execution plan (tb_netlist_plan): (levels [(row0, n_gates)], row_of_wire int64).  Level L's
+        outputs are rows row0 .. row0 + n_gates - 1 of the wire array (contiguous, as the all-gather needs)."""
+        s = self.c_struct()
+        nl = ctypes.c_int64(0)
+        _native.check(_native.lib().tb_netlist_plan(ctypes.byref(s), ctypes.byref(nl), None, None))
+        off = np.zeros(int(nl.value) + 1, np.int64)
+        rows = np.zeros(self.n_wires, np.int64)
+        _native.check(_native.lib().tb_netlist_plan(ctypes.byref(s), ctypes.byref(nl), off.ctypes.data,
+                                                    rows.ctypes.data))
+        levels = [(self.n_inputs + int(off[L]), int(off[L + 1] - off[L])) for L in range(int(nl.value))]
+        return levels, rows
+
 
 # ------------------------------------------------------------------------------------- binary format
 def _inst(hi62: int, mid62: int, t4: int) -> bytes:

@@ -1,0 +1,104 @@
+"""Multi-rank level loop on CPU (gloo, world sizes 2 and 3): sharding of each level, the padded in-place
+all-gather of output rows, and the wire layout from the native plan (tb_netlist_plan).  The per-gate work is
+a plaintext stand-in (the gate's truth table on bits), so this checks the distributed plumbing that the GPU
+path uses unchanged (paper_conf_ispass_maxw23_b200.parallel.level_loop); the kernels are covered by -m gpu.
+Expected values come from the oracle's plaintext simulator (oracle/plain.py).
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from oracle.plain import gate_bits, simulate
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _netlist(seed):
+    from test_host import random_dag
+    return random_dag(seed, n_inputs=7, n_gates=90)
+
+
+def _worker(rank, world, port, seed, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_ispass_maxw23_b200 as tb
+        from paper_conf_ispass_maxw23_b200 import parallel
+        n_in, t, a, b, c = _netlist(seed)
+        net = tb.Netlist(n_in, t, a, b, c)
+        levels, rows = net.plan()
+        order = np.argsort(rows[n_in:])                  # level-sorted position -> original gate index
+        bits = np.random.default_rng(seed).integers(0, 2, n_in).astype(np.int32)
+        slack = parallel.slack_rows(levels, net.n_wires, world)
+        wires = torch.full((net.n_wires + slack, 3), -1, dtype=torch.int32)
+        wires[:n_in, 0] = torch.from_numpy(bits)
+        calls = []
+
+        def run_level(L, g0, g1):
+            row0, ng = levels[L - 1]
+            calls.append((L, g0, g1))
+            for k in range(row0 - n_in + g0, row0 - n_in + g1):
+                g = order[k]
+                x = int(wires[rows[a[g]], 0])
+                y = int(wires[rows[b[g]], 0]) if t[g] != 3 else 0
+                z = int(wires[rows[c[g]], 0]) if t[g] == 16 else 0
+                wires[n_in + k, 0] = int(gate_bits(int(t[g]), x, y, z))
+                wires[n_in + k, 1] = rank                  # who computed it
+
+        parallel.level_loop(levels, wires, run_level, group=dist.group.WORLD)
+        q.put((rank, wires[:net.n_wires].numpy().copy(), calls, rows))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,seed", [(2, 1), (3, 2), (2, 5)])
+def test_level_loop_all_gather_matches_simulation(world, seed):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, seed, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    n_in, t, a, b, c = _netlist(seed)
+    bits = np.random.default_rng(seed).integers(0, 2, n_in)
+    want = simulate(n_in, t, a, b, c, bits)[0]
+    for rank, w, calls, rows in res:
+        assert (w[rows, 0] == want).all(), "rank %d wire values differ from the plaintext simulation" % rank
+    # every rank holds identical rows after the gathers, and each gate was computed by exactly one rank
+    ref = res[0][1]
+    for _, w, _, _ in res[1:]:
+        assert (w == ref).all()
+    owners = ref[n_in:, 1]
+    assert set(owners.tolist()) <= set(range(world))
+    computed = sorted(k for _, _, calls, _ in res for (L, g0, g1) in calls for k in range(g0, g1) for _ in [L])
+    assert len(computed) == len(t)
+
+
+def test_shard_and_slack():
+    from paper_conf_ispass_maxw23_b200 import parallel
+    assert parallel.shard(10, 4, 0) == (0, 3, 3) and parallel.shard(10, 4, 3) == (9, 10, 3)
+    assert parallel.shard(2, 4, 3) == (2, 2, 1)
+    assert parallel.shard(0, 8, 5) == (0, 0, 0)
+    # padded gather of the last level may run past n_rows by at most world*chunk - n_gates
+    assert parallel.slack_rows([(10, 10)], 20, 4) == 2
+    for ng in range(1, 50):
+        for R in (1, 2, 3, 8):
+            spans = [parallel.shard(ng, R, r) for r in range(R)]
+            assert sum(g1 - g0 for g0, g1, _ in spans) == ng
+            assert all(spans[r][1] == spans[r + 1][0] for r in range(R - 1))

@@ -1,0 +1,122 @@
+"""End-to-end netlists on the GPU (-m gpu): BASELINE configs[3] (VIP-Bench-shaped 32-bit multiplier,
+bubble sort) and configs[4] (ChiselTorch-shaped quantised MNIST Linear tile), plus sharded-level invariance.
+
+Parity at these sizes is (a) the decrypted outputs equal the plaintext function and (b) a seeded sample
+of gates is recomputed by the oracle from the GPU's own input wires and compared bit for bit (SURVEY 8(d):
+"per-gate local bit-exact parity on a seeded sample").  Whole-netlist oracle runs would take minutes.
+"""
+import numpy as np
+import pytest
+
+import oracle as O
+import synth
+from oracle.plain import simulate
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def tb():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import paper_conf_ispass_maxw23_b200 as tb
+    tb.build()
+    return tb
+
+
+@pytest.fixture(scope="module")
+def keys():
+    return O.keygen(O.DEFAULT, seed=77)
+
+
+@pytest.fixture(scope="module")
+def ctx(tb, keys):
+    c = tb.Context(0)
+    c.load_keys(keys.bk, keys.ksk)
+    return c
+
+
+def run(tb, ctx, n, cts):
+    net = tb.Netlist(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"], outputs=n["outputs"])
+    dnet = ctx.upload(net)
+    wires = ctx.wire_array(dnet)
+    wires[:net.n_inputs, :631] = ctx.to_device(cts)[:, :631]
+    ctx.run_netlist(dnet, wires)
+    return ctx.to_host(wires)[dnet.row_of_wire], dnet
+
+
+def sampled_gate_parity(keys, n, w, k, seed):
+    """recompute k seeded gates with the oracle from the GPU's own input wires"""
+    ng = len(n["type"])
+    idx = np.random.default_rng(seed).choice(ng, min(k, ng), replace=False)
+    ni = n["n_inputs"]
+    t = n["type"][idx]
+    a = w[n["in0"][idx]]
+    b = w[np.maximum(n["in1"][idx], 0)]
+    c = w[np.maximum(n["in2"][idx], 0)]
+    want = O.gates(keys, t, a, b, c)
+    assert (w[ni + idx] == want).all()
+    return idx
+
+
+def test_multiplier_32bit_config4(tb, ctx, keys):
+    n = synth.array_multiplier(32, full=True)
+    A, B = 0xDEADBEEF, 0x12345679
+    bits = np.concatenate([synth.pack_bits([A], 32), synth.pack_bits([B], 32)])
+    w, dnet = run(tb, ctx, n, O.encrypt_bits(keys, bits, 1))
+    dec = O.decrypt_bits(keys, w[n["outputs"]])
+    assert int(synth.unpack_bits(dec, 64)[0]) == A * B
+    plain = simulate(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"], bits)[0]
+    assert (O.decrypt_bits(keys, w) == plain).all()          # every wire decrypts to its plaintext
+    sampled_gate_parity(keys, n, w, 48, 2)
+
+
+def test_bubble_sort_config4(tb, ctx, keys):
+    n = synth.bubble_sort(8, 8)                                 # MUX-heavy, deep and narrow
+    vals = np.random.default_rng(3).integers(0, 256, 8)
+    bits = synth.pack_bits(vals, 8)
+    w, dnet = run(tb, ctx, n, O.encrypt_bits(keys, bits, 4))
+    dec = O.decrypt_bits(keys, w[n["outputs"]])
+    assert synth.unpack_bits(dec, 8).tolist() == sorted(vals.tolist())
+    idx = sampled_gate_parity(keys, n, w, 40, 5)
+    assert (n["type"] == O.MUX).any()
+
+
+def test_mnist_tile_config5(tb, ctx, keys):
+    n_in, n_out, bits_w = 8, 2, 8
+    n = synth.mnist_mlp_tile(n_in, n_out, bits_w)
+    rng = np.random.default_rng(6)
+    act, W = rng.integers(0, 256, n_in), rng.integers(0, 256, (n_out, n_in))
+    bits = np.concatenate([synth.pack_bits(act, 8), synth.pack_bits(W.reshape(-1), 8)])
+    w, dnet = run(tb, ctx, n, O.encrypt_bits(keys, bits, 7))
+    dec = O.decrypt_bits(keys, w[n["outputs"]])
+    width = len(n["outputs"]) // n_out
+    assert synth.unpack_bits(dec, width).tolist() == (W @ act).tolist()
+    sampled_gate_parity(keys, n, w, 40, 8)
+
+
+def test_sharded_levels_are_byte_identical(tb, ctx, keys):
+    """virtual ranks on one GPU: every level run as R shards [g0, g1) must give the same bytes as R = 1"""
+    n = synth.ripple_carry_adder(8)
+    n2 = synth.independent_level(37, 9)
+    for net_arrays in (n, n2):
+        cts = O.encrypt_bits(keys, synth.random_bits(net_arrays["n_inputs"], 10), 11)
+        ref, dnet = run(tb, ctx, net_arrays, cts)
+        for R in (2, 3, 8):
+            wires = ctx.wire_array(dnet)
+            wires[:net_arrays["n_inputs"], :631] = ctx.to_device(cts)[:, :631]
+            for L, (row0, ng, _, _) in enumerate(dnet.levels, start=1):
+                for r in range(R):
+                    g0, g1, _ = tb.parallel.shard(ng, R, r)
+                    ctx.run_level(dnet, L, g0, g1, wires)
+            got = ctx.to_host(wires)[dnet.row_of_wire]
+            assert (got == ref).all(), R
+
+
+def test_run_netlist_host_matches_device(tb, ctx, keys):
+    n = synth.ripple_carry_adder(4)
+    cts = O.encrypt_bits(keys, synth.random_bits(n["n_inputs"], 12), 13)
+    ref, dnet = run(tb, ctx, n, cts)
+    out = ctx.run_netlist_host(dnet, cts, n["outputs"])
+    assert (out == ref[n["outputs"]]).all()
