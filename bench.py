@@ -156,6 +156,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--gates-per-gpu", type=int, default=65536)
     ap.add_argument("--lanes-per-cta", type=int, default=2)
+    ap.add_argument("--br-variant", type=int, default=6, choices=[6, 7])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -185,6 +186,7 @@ def main():
     total = G * world
     ctx = tb.Context(local)
     ctx.set_lanes_per_cta(args.lanes_per_cta)
+    ctx.set_br_variant(args.br_variant)
     ctx.load_keys(synth.random_words(tb.BK_WORDS, 11), synth.random_words(tb.KSK_WORDS, 12))
     n = synth.independent_level(total, seed=13)
     net = tb.Netlist(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"], outputs=n["outputs"])
@@ -252,7 +254,7 @@ def main():
             traffic = None
     roofline = {"bound": "alu", "achieved": achieved / 1e9, "peak": peak / 1e9, "unit": "G IMAD-slots/s",
                 "frac": achieved / peak, "traffic": traffic,
-                "kernel": "br6_kernel (blind rotation + extraction)", "kernel_ms_per_launch": br_launch_s * 1e3,
+                "kernel": "br%d_kernel (blind rotation + extraction)" % args.br_variant, "kernel_ms_per_launch": br_launch_s * 1e3,
                 "kernel_share_of_step": br_ms / ms if ms else None,
                 "ks_kernel_ms_per_launch": ks_ms / max(ks_n, 1),
                 "peak_source": "derived: %d SMs x 64 IMAD lanes/clk x %.0f MHz (median SM clock in the timed region)"
@@ -317,7 +319,7 @@ def main():
             "data": "synthetic: seeded uniform key material and ciphertexts (evaluation is data-oblivious, P:160)",
             "config": {"workload": workload_name(G), "gates_per_gpu": G, "total_gates": total,
                        "parallelism": "dp%d (level sharded, NCCL all-gather of output rows)" % world,
-                       "lanes_per_cta": args.lanes_per_cta,
+                       "lanes_per_cta": args.lanes_per_cta, "br_variant": args.br_variant,
                        "l2": "inputs larger than L2 (%.0f MB of input ciphertexts per GPU)" % (2 * G * 2524 / 1e6)},
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
             "gpu_launches": br_n + ks_n,

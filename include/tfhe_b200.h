@@ -158,8 +158,12 @@ int tb_keyswitch(tb_ctx* ctx, const uint32_t* in, int64_t in_stride, uint32_t* o
  * digits [6][N] int32, polys [6][N] u32, res [N] u32.  Synchronous. */
 int tb_ntt_muladd6(tb_ctx* ctx, const int32_t* digits, const uint32_t* polys, uint32_t* res);
 
-/* Blind-rotation lanes per CTA (1..4, default 2); tuning knob, returns TB_EINVAL if out of range. */
+/* Blind-rotation lanes per CTA for the default kernel (1..4, default 2); tuning knob. */
 int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
+/* Blind-rotation kernel: 6 = br6_kernel (default: 6 warps/lane, 2 CTAs/SM, BK words from L2), 7 = br7_kernel
+ * (2 lanes/CTA, 1 CTA/SM, each 144 KB BK step TMA-bulk-copied into shared memory one step ahead).  Both are
+ * bit-identical; see DESIGN.md "Kernels". */
+int tb_set_br_variant(tb_ctx* ctx, int variant);
 /* Device bytes a context holds for keys (BK NTT + KSK). */
 int tb_key_bytes(const tb_ctx* ctx, size_t* bytes);
 

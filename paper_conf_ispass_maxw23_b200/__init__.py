@@ -118,6 +118,10 @@ class Context:
     def set_lanes_per_cta(self, lanes: int):
         _native.check(_native.lib().tb_set_lanes_per_cta(self._h, lanes))
 
+    def set_br_variant(self, variant: int):
+        """6 = br6_kernel (default), 7 = br7_kernel (TMA-staged BK); bit-identical outputs."""
+        _native.check(_native.lib().tb_set_br_variant(self._h, variant))
+
     # ---- tensors ----
     def empty(self, rows: int, stride: int = WIRE_STRIDE) -> torch.Tensor:
         return torch.empty((rows, stride), dtype=torch.int32, device=self.device)

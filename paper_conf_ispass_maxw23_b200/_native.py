@@ -87,6 +87,7 @@ SIGNATURES = {
     "tb_keyswitch": (ctypes.c_int, [_vp, _vp, _i64, _vp, _i64, _i64, _vp]),
     "tb_ntt_muladd6": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
     "tb_set_lanes_per_cta": (ctypes.c_int, [_vp, ctypes.c_int]),
+    "tb_set_br_variant": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_key_bytes": (ctypes.c_int, [_vp, ctypes.POINTER(_sz)]),
     "tb_microbench": (ctypes.c_int, [_vp, ctypes.c_int, ctypes.POINTER(ctypes.c_double),
                                      ctypes.POINTER(ctypes.c_double)]),

@@ -1,172 +1,14 @@
-// tb_bootstrap.cu -- the blind-rotation kernel and the BK -> NTT-domain kernel.
+// tb_bootstrap.cu -- load-time BK -> NTT-domain conversion and the tb_gates descriptor builder.
+// (The blind-rotation kernels themselves are in tb_br6.cu / tb_br7.cu.)
 //
-// PAPER.md: bootstrapping "dominates the execution time"; in a gate, blind rotation is the largest
-// slice (Fig. 7); its NTT work is "highly vectorizable" and independent gates "can be executed in
-// parallel".  This kernel therefore batches G independent bootstraps ("lanes") per CTA so that each
-// NTT-domain BK tile fetched for CMux step i feeds G accumulators, and runs all n = 630 CMux steps of those
-// lanes with the accumulators resident in shared memory (no HBM traffic for ACC).
-//
-// Per CTA: 2G warps.  Per CMux step i (for every lane g):
-//   phase A (warp (g, bloc)): T = (X^abar_i - 1) ACC[bloc]; 3 gadget digits of T (a4.1) -> 3 forward NTTs
-//   phase B (all threads)   : per NTT slot a: out[g][o][a] = sum_r D[g][r][a] * BKhat_i[r][o][a]  (a4.3)
-//   phase C (warp (g, q))   : 3 inverse NTTs (one per BK part), centred lift, recombine the parts,
-//                             ACC[q] += result (a4.4)
-// Exactness: DESIGN.md "Exactness" -- the integer result equals the schoolbook product mod 2^32 bit for bit.
+// The BK split used by every blind-rotation kernel: each torus coefficient
+// x = x0 + 2^11 x1 + 2^22 x2 (mod 2^32) with |x_m| <= 2^10, each part NTT-transformed mod p and pre-scaled by
+// N^-1, stored [i][r][o = q*3 + m][a].
 #include "tb_kernels.cuh"
 #include "tb_ntt.cuh"
 
 namespace tb {
 
-
-template <int G>
-struct BrSmem {
-    uint2 twF[31 * 32];
-    uint2 twI[31 * 32];
-    uint32_t acc[G][2][kN];
-    uint32_t slot[G][kOuts][kSlotWords];
-    uint16_t bar[G][kn + 2];
-};
-
-__device__ __forceinline__ const uint32_t* src_ptr(const BrArgs& A, uint32_t sel) {
-    return sel == 0 ? A.src0 : (sel == 1 ? A.src1 : A.src2);
-}
-
-template <int G>
-__global__ void __launch_bounds__(64 * G) br_kernel(BrArgs A) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    BrSmem<G>& S = *reinterpret_cast<BrSmem<G>*>(smem_raw);
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int lane0 = blockIdx.x * G;
-
-    for (int k = tid; k < 31 * 32; k += blockDim.x) {
-        S.twF[k] = A.twF[k];
-        S.twI[k] = A.twI[k];
-    }
-    // ---- prologue (a1, a2): linear gate combination + mod switch to 2N, one warp pair per lane ----
-    {
-        const int g = warp >> 1;
-        const int gl = lane0 + g;
-        LaneDesc d = {0, -1, 0, 0, 0u, 0u, 0u, 0u};
-        if (gl < A.nlanes) d = A.lanes[gl];
-        const uint32_t* pa = src_ptr(A, d.sel & 3u) + (int64_t)d.ia * A.src_stride;
-        const uint32_t* pb = d.ib >= 0 ? src_ptr(A, (d.sel >> 2) & 3u) + (int64_t)d.ib * A.src_stride : nullptr;
-        for (int w = (warp & 1) * 32 + lane; w <= kn; w += 64) {
-            uint32_t v = (gl < A.nlanes) ? (uint32_t)d.wa * __ldg(pa + w) : 0u;
-            if (pb) v += (uint32_t)d.wb * __ldg(pb + w);
-            if (w == kn) v += d.cst;
-            S.bar[g][w] = (uint16_t)((v + (1u << 20)) >> 21);      // round(v 2N / 2^32) mod 2N (C5)
-        }
-    }
-    __syncthreads();
-    // ---- ACC = (0, X^{-bbar} (mu, ..., mu))  (a3, C6) ----
-    for (int k = tid; k < G * kN; k += blockDim.x) {
-        const int g = k / kN, c = k % kN;
-        const uint32_t bbar = S.bar[g][kn];
-        S.acc[g][0][c] = 0u;
-        S.acc[g][1][c] = ((c + bbar) & (kTwoN - 1)) < (uint32_t)kN ? kMu : (uint32_t)(0u - kMu);
-    }
-    __syncthreads();
-
-    const uint32_t R = c_misc[0], Rp = c_misc[1];
-    for (int i = 0; i < kn; i++) {
-        // ---- phase A: rotate, decompose, forward NTT (a4.1, a4.2) ----
-        {
-            const int g = warp >> 1, bloc = warp & 1;
-            const uint32_t ab = S.bar[g][i];
-            const uint32_t* acc = S.acc[g][bloc];
-            uint32_t U[32];
-#pragma unroll
-            for (int j = 0; j < 32; j++) {
-                const uint32_t c = lane + 32 * j;
-                const uint32_t m = (c - ab) & (kTwoN - 1);            // X^ab ACC: coefficient c
-                const uint32_t src = acc[m & (kN - 1)];
-                const uint32_t rot = m < (uint32_t)kN ? src : 0u - src;
-                U[j] = rot - acc[c] + kDecompOffset;                    // (X^ab - 1) ACC + offset
-            }
-#pragma unroll
-            for (int jd = 0; jd < kL; jd++) {
-                uint32_t x[32];
-#pragma unroll
-                for (int j = 0; j < 32; j++)                             // digit in [-64, 63], as mod p
-                    x[j] = ((U[j] >> (32 - kBgbit * (jd + 1))) & 127u) + (kP - 64u);
-                uint32_t* slot = S.slot[g][bloc * kL + jd];
-                ntt_fwd(x, slot, S.twF, lane);
-#pragma unroll
-                for (int j = 0; j < 32; j++) slot[kPadRow * lane + j] = red_2p(x[j]);
-            }
-        }
-        __syncthreads();
-        // ---- phase B: pointwise MAC against the NTT-domain BK_i, shared by the CTA's G lanes (a4.3) ----
-        {
-            const uint32_t* bki = A.bkhat + (size_t)i * (kRows * kOuts * kN);
-            for (int a = tid; a < kN; a += 64 * G) {
-                const int pa = a + (a >> 5);
-                uint64_t acc[G][kOuts];
-#pragma unroll
-                for (int g = 0; g < G; g++)
-#pragma unroll
-                    for (int o = 0; o < kOuts; o++) acc[g][o] = 0ull;
-#pragma unroll
-                for (int r = 0; r < kRows; r++) {
-                    uint32_t B[kOuts];
-#pragma unroll
-                    for (int o = 0; o < kOuts; o++) B[o] = __ldg(bki + (r * kOuts + o) * kN + a);
-#pragma unroll
-                    for (int g = 0; g < G; g++) {
-                        const uint32_t dv = S.slot[g][r][pa];
-#pragma unroll
-                        for (int o = 0; o < kOuts; o++) acc[g][o] += (uint64_t)dv * B[o];
-                    }
-                }
-#pragma unroll
-                for (int g = 0; g < G; g++)
-#pragma unroll
-                    for (int o = 0; o < kOuts; o++) {
-                        const uint32_t hi = (uint32_t)(acc[g][o] >> 32), lo = (uint32_t)acc[g][o];
-                        const uint32_t v = shoup_mul(hi, R, Rp) + (lo - (lo >> 30) * kP);   // < 4p
-                        S.slot[g][o][pa] = red_2p(v);
-                    }
-            }
-        }
-        __syncthreads();
-        // ---- phase C: inverse NTTs, centred lift, part recombination, ACC += (a4.4) ----
-        {
-            const int g = warp >> 1, q = warp & 1;
-            uint32_t sum[32];
-#pragma unroll
-            for (int j = 0; j < 32; j++) sum[j] = 0u;
-#pragma unroll
-            for (int m = 0; m < kParts; m++) {
-                uint32_t* slot = S.slot[g][q * kParts + m];
-                uint32_t x[32];
-#pragma unroll
-                for (int j = 0; j < 32; j++) x[j] = slot[kPadRow * lane + j];
-                ntt_inv(x, slot, S.twI, lane);
-#pragma unroll
-                for (int j = 0; j < 32; j++) sum[j] += lift_centred(x[j]) << (11 * m);
-            }
-            uint32_t* acc = S.acc[g][q];
-#pragma unroll
-            for (int j = 0; j < 32; j++) acc[lane + 32 * j] += sum[j];
-        }
-        __syncthreads();
-    }
-    // ---- sample extraction, index 0 (a5, C8) ----
-    {
-        const int g = warp >> 1;
-        const int gl = lane0 + g;
-        if (gl < A.nlanes) {
-            uint32_t* o = A.out + (int64_t)gl * A.out_stride;
-            for (int j = (warp & 1) * 32 + lane; j <= kN; j += 64) {
-                uint32_t v;
-                if (j == 0) v = S.acc[g][0][0];
-                else if (j < kN) v = 0u - S.acc[g][0][kN - j];
-                else v = S.acc[g][1][0];
-                o[j] = v;
-            }
-        }
-    }
-}
 
 // ---------------------------------------------------------------------------------------------------
 // BK (torus, [n][6][2][N] u32) -> NTT domain [n][6][6][N]: each coefficient split into 3 signed parts
@@ -235,41 +77,6 @@ __global__ void build_gate_desc_kernel(int gate_kind, int32_t wa, int32_t wb, ui
 
 // ---------------------------------------------------------------------------------------------------
 // host-side launchers (C++ linkage, used by tb_runtime.cu)
-template <int G>
-static int launch_br_g(const BrArgs& A, cudaStream_t st) {
-    const size_t smem = sizeof(BrSmem<G>);
-    static bool attr = false;
-    if (!attr) {
-        if (cudaFuncSetAttribute(br_kernel<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
-            return -1;
-        attr = true;
-    }
-    const int blocks = (A.nlanes + G - 1) / G;
-    if (blocks == 0) return 0;
-    br_kernel<G><<<blocks, 64 * G, smem, st>>>(A);
-    return 0;
-}
-
-int launch_br(const BrArgs& A, int G, cudaStream_t st) {
-    switch (G) {
-        case 1: return launch_br_g<1>(A, st);
-        case 2: return launch_br_g<2>(A, st);
-        case 3: return launch_br_g<3>(A, st);
-        case 4: return launch_br_g<4>(A, st);
-        default: return -2;
-    }
-}
-
-size_t br_smem_bytes(int G) {
-    switch (G) {
-        case 1: return sizeof(BrSmem<1>);
-        case 2: return sizeof(BrSmem<2>);
-        case 3: return sizeof(BrSmem<3>);
-        case 4: return sizeof(BrSmem<4>);
-        default: return 0;
-    }
-}
-
 void launch_bk_to_ntt(const uint32_t* bk, uint32_t* bkhat, const uint2* twF, uint32_t ninv, uint32_t ninvp,
                       cudaStream_t st) {
     const int tasks = kn * kRows * 2 * kParts;

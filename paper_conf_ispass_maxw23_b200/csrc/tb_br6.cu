@@ -1,7 +1,11 @@
-// tb_br6.cu -- blind rotation, six warps per lane.
+// tb_br6.cu -- the blind-rotation kernel, six warps per lane.
 //
-// Same arithmetic as br_kernel (tb_bootstrap.cu) -- bit-identical output -- with the work of one CMux step
-// spread over 6 warps per lane (one transform per warp) so that an SM holds 24 warps (2 CTAs x 2 lanes x 6):
+// PAPER.md: bootstrapping "dominates the execution time"; in a gate, blind rotation is the largest
+// slice (Fig. 7); its NTT work is "highly vectorizable" and independent gates "can be executed in
+// parallel".  A CTA therefore batches G independent bootstraps ("lanes") so that each NTT-domain BK
+// word fetched for CMux step i feeds G accumulators, and runs all n = 630 CMux steps of those lanes with the
+// accumulators resident in shared memory.  The work of one CMux step is spread over 6 warps per lane (one
+// transform per warp) so that an SM holds 24 warps (2 CTAs x 2 lanes x 6):
 //   phase A (warp (g, r), r = bloc*l + jd): digit jd of (X^abar - 1) ACC[bloc] -> forward NTT -> slot r
 //   phase B (all threads, one coefficient a per item): the 36 BK_i words of a are loaded at once (MLP for
 //           the L2 latency), out[g][o][a] = sum_r D[g][r][a] BKhat_i[r][o][a], written back in place
@@ -27,7 +31,7 @@ __device__ __forceinline__ void named_bar(int id, int nthreads) {
 
 template <int G>
 __global__ void __launch_bounds__(192 * G, (G <= 2 ? 2 : 1)) br6_kernel(BrArgs A) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
+    extern __shared__ __align__(128) unsigned char smem_raw[];
     Br6Smem<G>& S = *reinterpret_cast<Br6Smem<G>*>(smem_raw);
     constexpr int NT = 192 * G;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;

@@ -28,7 +28,7 @@ struct DiagSmem {
 __global__ void __launch_bounds__(192) ntt_muladd6_kernel(const int32_t* digits, const uint32_t* polys,
                                                           uint32_t* res, const uint2* twF, const uint2* twI,
                                                           uint32_t ninv, uint32_t ninvp) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
+    extern __shared__ __align__(128) unsigned char smem_raw[];
     DiagSmem& S = *reinterpret_cast<DiagSmem*>(smem_raw);
     const int lane = threadIdx.x & 31, r = threadIdx.x >> 5;
     for (int k = threadIdx.x; k < 31 * 32; k += blockDim.x) {

@@ -29,6 +29,13 @@ __device__ __forceinline__ uint32_t shoup_mul(uint32_t y, uint32_t w, uint32_t w
 __device__ __forceinline__ uint32_t red_2p(uint32_t x) { return min(x, x - kTwoP); }  // [0,4p) -> [0,2p)
 __device__ __forceinline__ uint32_t red_p(uint32_t x) { return min(x, x - kP); }      // [0,2p) -> [0,p)
 
+// element (row, col) of a 32x32 transpose buffer: padded rows of 33 words, or 32-word rows with the column
+// XOR-swizzled by the row (both conflict-free for row-wise and column-wise warp access)
+template <bool SWZ>
+__device__ __forceinline__ int sidx(int row, int col) {
+    return SWZ ? ((row << 5) | (col ^ row)) : row * kPadRow + col;
+}
+
 // CT butterfly, inputs and outputs in [0, 4p)
 __device__ __forceinline__ void ct_bfly(uint32_t& x, uint32_t& y, uint32_t w, uint32_t wp) {
     const uint32_t X = red_2p(x);
@@ -46,6 +53,7 @@ __device__ __forceinline__ void gs_bfly(uint32_t& x, uint32_t& y, uint32_t w, ui
 
 // Forward NTT.  In: x[j] = a[lane + 32 j] (< 4p).  Out: x[j] = A[32 lane + j] (< 4p).
 // buf: warp-private 32x33 shared buffer.  twT: shared per-lane twiddle table [31][32] (w, w').
+template <bool SWZ = false>
 __device__ __forceinline__ void ntt_fwd(uint32_t (&x)[32], uint32_t* buf, const uint2* twT, int lane) {
 #pragma unroll
     for (int s = 0; s < 5; s++) {
@@ -58,10 +66,10 @@ __device__ __forceinline__ void ntt_fwd(uint32_t (&x)[32], uint32_t* buf, const 
         }
     }
 #pragma unroll
-    for (int j = 0; j < 32; j++) buf[kPadRow * j + lane] = x[j];
+    for (int j = 0; j < 32; j++) buf[sidx<SWZ>(j, lane)] = x[j];
     __syncwarp();
 #pragma unroll
-    for (int j = 0; j < 32; j++) x[j] = buf[kPadRow * lane + j];
+    for (int j = 0; j < 32; j++) x[j] = buf[sidx<SWZ>(lane, j)];
 #pragma unroll
     for (int s = 5; s < 10; s++) {
         const int len = 16 >> (s - 5);
@@ -75,6 +83,7 @@ __device__ __forceinline__ void ntt_fwd(uint32_t (&x)[32], uint32_t* buf, const 
 }
 
 // Inverse NTT (without the 1/N factor).  In: x[j] = A[32 lane + j] (< 2p).  Out: x[j] = N a[lane + 32 j] (< 2p).
+template <bool SWZ = false>
 __device__ __forceinline__ void ntt_inv(uint32_t (&x)[32], uint32_t* buf, const uint2* twTi, int lane) {
 #pragma unroll
     for (int s = 9; s >= 5; s--) {
@@ -88,10 +97,10 @@ __device__ __forceinline__ void ntt_inv(uint32_t (&x)[32], uint32_t* buf, const 
     }
     __syncwarp();
 #pragma unroll
-    for (int j = 0; j < 32; j++) buf[kPadRow * lane + j] = x[j];
+    for (int j = 0; j < 32; j++) buf[sidx<SWZ>(lane, j)] = x[j];
     __syncwarp();
 #pragma unroll
-    for (int j = 0; j < 32; j++) x[j] = buf[kPadRow * j + lane];
+    for (int j = 0; j < 32; j++) x[j] = buf[sidx<SWZ>(j, lane)];
 #pragma unroll
     for (int s = 4; s >= 0; s--) {
         const int len = 16 >> s;

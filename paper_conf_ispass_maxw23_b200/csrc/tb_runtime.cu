@@ -59,7 +59,7 @@ static uint32_t brv10(uint32_t k) {
 struct tb_ctx {
     int device = 0;
     int lanes_per_cta = 2;
-    int variant = 6;                        // blind-rotation kernel: 6 = br6_kernel (6 warps/lane), 2 = br_kernel
+    int variant = 6;                        // blind-rotation kernel: 6 = br6_kernel, 7 = br7_kernel (TMA-staged BK)
     cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
     uint2* twF = nullptr;                   // [31][32]
     uint2* twI = nullptr;
@@ -170,7 +170,6 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
     tb_ctx* c = new (std::nothrow) tb_ctx();
     if (!c) return fail(TB_ENOMEM, "host allocation failed");
     c->device = dev;
-    if (const char* v = getenv("TB_BR_VARIANT")) c->variant = atoi(v);   // experiment knob (6 or 2)
 
     // psi: primitive 2N-th root of unity mod p (psi^N = -1)
     uint32_t psi = 0;
@@ -237,6 +236,12 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
 extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
     if (!c || lanes < 1 || lanes > 4) return fail(TB_EINVAL, "lanes per CTA must be 1..4");
     c->lanes_per_cta = lanes;
+    return TB_OK;
+}
+
+extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
+    if (!c || (variant != 6 && variant != 7)) return fail(TB_EINVAL, "blind-rotation variant must be 6 or 7");
+    c->variant = variant;
     return TB_OK;
 }
 
@@ -324,7 +329,7 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     A.lanes = lanes; A.nlanes = (int32_t)nlanes; A.bkhat = c->bkhat; A.twF = c->twF; A.twI = c->twI;
     A.out = out; A.out_stride = ostride;
     const long slot = prof_begin(c, 0, st);
-    int rc = c->variant == 6 ? launch_br6(A, c->lanes_per_cta, st) : launch_br(A, c->lanes_per_cta, st);
+    int rc = c->variant == 7 ? launch_br7(A, st) : launch_br6(A, c->lanes_per_cta, st);
     prof_end(c, slot, st);
     if (rc) return fail(TB_ECUDA, "blind-rotation kernel attribute/launch failed");
     cudaError_t e = cudaGetLastError();
