@@ -164,6 +164,8 @@ int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
  * (2 lanes/CTA, 1 CTA/SM, each 144 KB BK step TMA-bulk-copied into shared memory one step ahead).  Both are
  * bit-identical; see DESIGN.md "Kernels". */
 int tb_set_br_variant(tb_ctx* ctx, int variant);
+/* Gates per key-switch CTA (8, 16 or 32; default 8): each tile streams the 62 MB KSK once from L2. */
+int tb_set_ks_tile(tb_ctx* ctx, int gates);
 /* Device bytes a context holds for keys (BK NTT + KSK). */
 int tb_key_bytes(const tb_ctx* ctx, size_t* bytes);
 

@@ -122,6 +122,10 @@ class Context:
         """6 = br6_kernel (default), 7 = br7_kernel (TMA-staged BK); bit-identical outputs."""
         _native.check(_native.lib().tb_set_br_variant(self._h, variant))
 
+    def set_ks_tile(self, gates: int):
+        """gates per key-switch CTA: 8 (default), 16 or 32"""
+        _native.check(_native.lib().tb_set_ks_tile(self._h, gates))
+
     # ---- tensors ----
     def empty(self, rows: int, stride: int = WIRE_STRIDE) -> torch.Tensor:
         return torch.empty((rows, stride), dtype=torch.int32, device=self.device)

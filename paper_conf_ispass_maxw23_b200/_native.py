@@ -88,6 +88,7 @@ SIGNATURES = {
     "tb_ntt_muladd6": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
     "tb_set_lanes_per_cta": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_set_br_variant": (ctypes.c_int, [_vp, ctypes.c_int]),
+    "tb_set_ks_tile": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_key_bytes": (ctypes.c_int, [_vp, ctypes.POINTER(_sz)]),
     "tb_microbench": (ctypes.c_int, [_vp, ctypes.c_int, ctypes.POINTER(ctypes.c_double),
                                      ctypes.POINTER(ctypes.c_double)]),

@@ -15,8 +15,9 @@ constexpr int kKsThreads = 160;                  // 158 threads x 4 words = 632 
 
 template <int T>
 __global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A) {
-    __shared__ __align__(16) uint16_t sW[kN][T];  // (a_i + 2^15) >> 16: all 8 digits of a_i
-    __shared__ uint32_t sB[T];
+    extern __shared__ __align__(128) unsigned char ks_smem[];
+    uint16_t (*sW)[T] = reinterpret_cast<uint16_t (*)[T]>(ks_smem);   // [kN][T]: (a_i + 2^15) >> 16 = 8 digits
+    uint32_t* sB = reinterpret_cast<uint32_t*>(ks_smem + (size_t)kN * T * 2);
     const int tid = threadIdx.x;
     const int g0 = blockIdx.x * T;
 
@@ -102,13 +103,28 @@ __global__ void ksk_relayout_kernel(const uint32_t* __restrict__ src, uint32_t* 
     for (int k = threadIdx.x; k < kKsRow; k += blockDim.x) d[k] = k <= kn ? s[k] : 0u;
 }
 
-constexpr int kKsTile = 16;
-
-int launch_ks(const KsArgs& A, cudaStream_t st) {
-    if (A.ngates <= 0) return 0;
-    const int blocks = (A.ngates + kKsTile - 1) / kKsTile;
-    ks_kernel<kKsTile><<<blocks, kKsThreads, 0, st>>>(A);
+template <int T>
+static int launch_ks_t(const KsArgs& A, cudaStream_t st) {
+    const size_t smem = (size_t)kN * T * 2 + T * 4;
+    static bool attr = false;
+    if (!attr) {
+        if (cudaFuncSetAttribute(ks_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+            return -1;
+        attr = true;
+    }
+    const int blocks = (A.ngates + T - 1) / T;
+    ks_kernel<T><<<blocks, kKsThreads, smem, st>>>(A);
     return 0;
+}
+
+int launch_ks(const KsArgs& A, int tile, cudaStream_t st) {
+    if (A.ngates <= 0) return 0;
+    switch (tile) {
+        case 8: return launch_ks_t<8>(A, st);
+        case 16: return launch_ks_t<16>(A, st);
+        case 32: return launch_ks_t<32>(A, st);
+        default: return -2;
+    }
 }
 
 void launch_ksk_relayout(const uint32_t* src, uint32_t* dst, cudaStream_t st) {

@@ -59,7 +59,8 @@ static uint32_t brv10(uint32_t k) {
 struct tb_ctx {
     int device = 0;
     int lanes_per_cta = 2;
-    int variant = 6;                        // blind-rotation kernel: 6 = br6_kernel, 7 = br7_kernel (TMA-staged BK)
+    int variant = 6;                        // blind-rotation kernel: 6 = br6, 7 = br7 (TMA-staged BK), 8 = br8
+    int ks_tile = 8;                        // gates per key-switch CTA (8, 16, 32); 8 measured fastest
     cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
     uint2* twF = nullptr;                   // [31][32]
     uint2* twI = nullptr;
@@ -240,8 +241,14 @@ extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
 }
 
 extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
-    if (!c || (variant != 6 && variant != 7)) return fail(TB_EINVAL, "blind-rotation variant must be 6 or 7");
+    if (!c || variant < 6 || variant > 8) return fail(TB_EINVAL, "blind-rotation variant must be 6, 7 or 8");
     c->variant = variant;
+    return TB_OK;
+}
+
+extern "C" int tb_set_ks_tile(tb_ctx* c, int gates) {
+    if (!c || (gates != 8 && gates != 16 && gates != 32)) return fail(TB_EINVAL, "key-switch tile must be 8, 16 or 32");
+    c->ks_tile = gates;
     return TB_OK;
 }
 
@@ -329,7 +336,8 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     A.lanes = lanes; A.nlanes = (int32_t)nlanes; A.bkhat = c->bkhat; A.twF = c->twF; A.twI = c->twI;
     A.out = out; A.out_stride = ostride;
     const long slot = prof_begin(c, 0, st);
-    int rc = c->variant == 7 ? launch_br7(A, st) : launch_br6(A, c->lanes_per_cta, st);
+    int rc = c->variant == 7 ? launch_br7(A, st)
+             : c->variant == 8 ? launch_br8(A, st) : launch_br6(A, c->lanes_per_cta, st);
     prof_end(c, slot, st);
     if (rc) return fail(TB_ECUDA, "blind-rotation kernel attribute/launch failed");
     cudaError_t e = cudaGetLastError();
@@ -345,7 +353,7 @@ static int run_ks(tb_ctx* c, const uint32_t* lanes, int64_t lane_base, int64_t l
     A.ngates = (int32_t)ngates; A.ksk = c->ksk; A.out = out; A.out_stride = ostride; A.not_src = not_src;
     A.not_stride = not_stride;
     const long slot = prof_begin(c, 1, st);
-    launch_ks(A, st);
+    if (launch_ks(A, c->ks_tile, st)) return fail(TB_ECUDA, "key-switch kernel attribute/launch failed");
     prof_end(c, slot, st);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "ks_kernel launch");

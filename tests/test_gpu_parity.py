@@ -71,6 +71,20 @@ def test_bootstrap_wo_ks_bit_exact(tb, ctx, keys):
         assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), k
 
 
+@pytest.mark.parametrize("variant", [6, 7, 8])
+def test_blind_rotation_variants_bit_exact(tb, ctx, keys, variant):
+    """every blind-rotation kernel variant (br6 / br7 TMA-staged / br8 ping-pong) on a ragged batch of 9"""
+    rng = np.random.default_rng(40 + variant)
+    cts = rng.integers(0, M32, (9, 631), dtype=np.uint64).astype(np.uint32)
+    ctx.set_br_variant(variant)
+    try:
+        got = ctx.bootstrap_wo_ks(ctx.to_device(cts))[:, :1025].cpu().numpy().view(np.uint32)
+    finally:
+        ctx.set_br_variant(6)
+    for k in range(9):
+        assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), k
+
+
 def test_trivial_inputs_closed_form(tb, ctx):
     phis = [0, 1, (1 << 20) - 1, 1 << 20, 1 << 31, M32 - (1 << 20) - 1, M32 - (1 << 20), M32 - 1, 0x9E3779B9]
     cts = np.zeros((len(phis), 631), np.uint32)
