@@ -178,6 +178,7 @@ def main():
     import paper_conf_ispass_maxw23_b200 as tb
     import synth
 
+    tb.build()                                        # no-op when the in-tree .so is current
     torch.cuda.set_device(local)
     group = None
     if world > 1:

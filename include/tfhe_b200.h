@@ -164,6 +164,9 @@ int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
  * (2 lanes/CTA, 1 CTA/SM, each 144 KB BK step TMA-bulk-copied into shared memory one step ahead).  Both are
  * bit-identical; see DESIGN.md "Kernels". */
 int tb_set_br_variant(tb_ctx* ctx, int variant);
+/* Latency mode for narrow levels: a launch with <= `lanes` bootstraps uses br7 with one lane per CTA (one
+ * SM per bootstrap, BK step staged in shared memory).  Default = the device's SM count; 0 disables. */
+int tb_set_narrow_lanes(tb_ctx* ctx, int64_t lanes);
 /* Gates per key-switch CTA (8, 16 or 32; default 8): each tile streams the 62 MB KSK once from L2. */
 int tb_set_ks_tile(tb_ctx* ctx, int gates);
 /* Device bytes a context holds for keys (BK NTT + KSK). */

@@ -122,6 +122,10 @@ class Context:
         """6 = br6_kernel (default), 7 = br7_kernel (TMA-staged BK); bit-identical outputs."""
         _native.check(_native.lib().tb_set_br_variant(self._h, variant))
 
+    def set_narrow_lanes(self, lanes: int):
+        """levels with <= lanes bootstraps run in latency mode (br7, one lane per SM); 0 disables"""
+        _native.check(_native.lib().tb_set_narrow_lanes(self._h, lanes))
+
     def set_ks_tile(self, gates: int):
         """gates per key-switch CTA: 8 (default), 16 or 32"""
         _native.check(_native.lib().tb_set_ks_tile(self._h, gates))

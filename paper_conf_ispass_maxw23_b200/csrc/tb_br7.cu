@@ -14,13 +14,14 @@ namespace tb {
 
 constexpr int kBkStepWords = kRows * kOuts * kN;          // 36,864 words = 147,456 B per CMux step
 
+template <int G>
 struct __align__(128) Br7Smem {
     uint32_t bk[kBkStepWords];
     uint2 twF[31 * 32];
     uint2 twI[31 * 32];
-    uint32_t acc[2][2][kN];
-    uint32_t slot[2][kOuts][32 * 32];
-    uint16_t bar[2][kn + 2];
+    uint32_t acc[G][2][kN];
+    uint32_t slot[G][kOuts][32 * 32];
+    uint16_t bar[G][kn + 2];
     unsigned long long mbar;
 };
 
@@ -46,7 +47,8 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
                  : "memory");
 }
 // one thread: request BK_i (6 bulk copies of 24 KB) on the CTA's mbarrier
-__device__ __forceinline__ void issue_bk(Br7Smem& S, const uint32_t* bkhat, int i) {
+template <int G>
+__device__ __forceinline__ void issue_bk(Br7Smem<G>& S, const uint32_t* bkhat, int i) {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // prior generic reads of S.bk are done
     mbar_expect_tx(&S.mbar, kBkStepWords * 4);
     const uint32_t* src = bkhat + (size_t)i * kBkStepWords;
@@ -59,10 +61,11 @@ __device__ __forceinline__ void named_bar7(int id, int nthreads) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-__global__ void __launch_bounds__(384, 1) br7_kernel(BrArgs A) {
+template <int G>
+__global__ void __launch_bounds__(192 * G, 1) br7_kernel(BrArgs A) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
-    Br7Smem& S = *reinterpret_cast<Br7Smem*>(smem_raw);
-    constexpr int G = 2, NT = 384;
+    Br7Smem<G>& S = *reinterpret_cast<Br7Smem<G>*>(smem_raw);
+    constexpr int NT = 192 * G;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int g = warp / 6, w6 = warp % 6;
     const int lane0 = blockIdx.x * G;
@@ -139,18 +142,20 @@ __global__ void __launch_bounds__(384, 1) br7_kernel(BrArgs A) {
                 for (int r = 0; r < kRows; r++) D[gg][r] = S.slot[gg][r][sa];
 #pragma unroll
             for (int o = 0; o < kOuts; o++) {
-                uint64_t s0 = 0, s1 = 0;
+                uint64_t s[G];
+#pragma unroll
+                for (int gg = 0; gg < G; gg++) s[gg] = 0;
 #pragma unroll
                 for (int r = 0; r < kRows; r++) {
                     const uint32_t b = S.bk[(r * kOuts + o) * kN + a];
-                    s0 += (uint64_t)D[0][r] * b;
-                    s1 += (uint64_t)D[1][r] * b;
+#pragma unroll
+                    for (int gg = 0; gg < G; gg++) s[gg] += (uint64_t)D[gg][r] * b;
                 }
-                uint32_t hi = (uint32_t)(s0 >> 32), lo = (uint32_t)s0;
-                S.slot[0][o][sa] = red_2p(shoup_mul(hi, R, Rp) + (lo - (lo >> 30) * kP));
-                hi = (uint32_t)(s1 >> 32);
-                lo = (uint32_t)s1;
-                S.slot[1][o][sa] = red_2p(shoup_mul(hi, R, Rp) + (lo - (lo >> 30) * kP));
+#pragma unroll
+                for (int gg = 0; gg < G; gg++) {
+                    const uint32_t hi = (uint32_t)(s[gg] >> 32), lo = (uint32_t)s[gg];
+                    S.slot[gg][o][sa] = red_2p(shoup_mul(hi, R, Rp) + (lo - (lo >> 30) * kP));
+                }
             }
         }
         __syncthreads();
@@ -195,18 +200,25 @@ __global__ void __launch_bounds__(384, 1) br7_kernel(BrArgs A) {
     }
 }
 
-int launch_br7(const BrArgs& A, cudaStream_t st) {
-    const size_t smem = sizeof(Br7Smem);
+template <int G>
+static int launch_br7_g(const BrArgs& A, cudaStream_t st) {
+    const size_t smem = sizeof(Br7Smem<G>);
     static bool attr = false;
     if (!attr) {
-        if (cudaFuncSetAttribute(br7_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+        if (cudaFuncSetAttribute(br7_kernel<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+            cudaSuccess)
             return -1;
         attr = true;
     }
-    const int blocks = (A.nlanes + 1) / 2;
+    const int blocks = (A.nlanes + G - 1) / G;
     if (blocks == 0) return 0;
-    br7_kernel<<<blocks, 384, smem, st>>>(A);
+    br7_kernel<G><<<blocks, 192 * G, smem, st>>>(A);
     return 0;
+}
+
+// G = 2: throughput variant; G = 1: latency mode for narrow levels (one lane per SM, BK staged per step)
+int launch_br7(const BrArgs& A, int G, cudaStream_t st) {
+    return G == 1 ? launch_br7_g<1>(A, st) : launch_br7_g<2>(A, st);
 }
 
 }  // namespace tb

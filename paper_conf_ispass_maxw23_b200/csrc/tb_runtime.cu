@@ -61,6 +61,7 @@ struct tb_ctx {
     int lanes_per_cta = 2;
     int variant = 6;                        // blind-rotation kernel: 6 = br6, 7 = br7 (TMA-staged BK), 8 = br8
     int ks_tile = 8;                        // gates per key-switch CTA (8, 16, 32); 8 measured fastest
+    int narrow_lanes = 0;                   // levels with <= this many lanes use br7<1> (set to the SM count)
     cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
     uint2* twF = nullptr;                   // [31][32]
     uint2* twI = nullptr;
@@ -171,6 +172,7 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
     tb_ctx* c = new (std::nothrow) tb_ctx();
     if (!c) return fail(TB_ENOMEM, "host allocation failed");
     c->device = dev;
+    c->narrow_lanes = prop.multiProcessorCount;
 
     // psi: primitive 2N-th root of unity mod p (psi^N = -1)
     uint32_t psi = 0;
@@ -243,6 +245,12 @@ extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
 extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
     if (!c || variant < 6 || variant > 8) return fail(TB_EINVAL, "blind-rotation variant must be 6, 7 or 8");
     c->variant = variant;
+    return TB_OK;
+}
+
+extern "C" int tb_set_narrow_lanes(tb_ctx* c, int64_t lanes) {
+    if (!c || lanes < 0) return fail(TB_EINVAL, "narrow-level threshold must be >= 0");
+    c->narrow_lanes = lanes;
     return TB_OK;
 }
 
@@ -336,8 +344,15 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     A.lanes = lanes; A.nlanes = (int32_t)nlanes; A.bkhat = c->bkhat; A.twF = c->twF; A.twI = c->twI;
     A.out = out; A.out_stride = ostride;
     const long slot = prof_begin(c, 0, st);
-    int rc = c->variant == 7 ? launch_br7(A, st)
-             : c->variant == 8 ? launch_br8(A, st) : launch_br6(A, c->lanes_per_cta, st);
+    int rc;
+    if (c->narrow_lanes > 0 && nlanes <= c->narrow_lanes)
+        rc = launch_br7(A, 1, st);                      // narrow level: one lane per SM, BK staged per step
+    else if (c->variant == 7)
+        rc = launch_br7(A, 2, st);
+    else if (c->variant == 8)
+        rc = launch_br8(A, st);
+    else
+        rc = launch_br6(A, c->lanes_per_cta, st);
     prof_end(c, slot, st);
     if (rc) return fail(TB_ECUDA, "blind-rotation kernel attribute/launch failed");
     cudaError_t e = cudaGetLastError();

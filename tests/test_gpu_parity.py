@@ -71,16 +71,28 @@ def test_bootstrap_wo_ks_bit_exact(tb, ctx, keys):
         assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), k
 
 
+def test_narrow_level_latency_mode_bit_exact(tb, ctx, keys):
+    """small launches run br7<1> (one lane per SM); 149 lanes fall back to the throughput kernel"""
+    rng = np.random.default_rng(39)
+    for count in (1, 3, 149):
+        cts = rng.integers(0, M32, (count, 631), dtype=np.uint64).astype(np.uint32)
+        got = ctx.bootstrap_wo_ks(ctx.to_device(cts))[:, :1025].cpu().numpy().view(np.uint32)
+        for k in sorted({0, count - 1}):
+            assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), (count, k)
+
+
 @pytest.mark.parametrize("variant", [6, 7, 8])
 def test_blind_rotation_variants_bit_exact(tb, ctx, keys, variant):
     """every blind-rotation kernel variant (br6 / br7 TMA-staged / br8 ping-pong) on a ragged batch of 9"""
     rng = np.random.default_rng(40 + variant)
     cts = rng.integers(0, M32, (9, 631), dtype=np.uint64).astype(np.uint32)
     ctx.set_br_variant(variant)
+    ctx.set_narrow_lanes(0)                  # throughput kernels even for a small batch
     try:
         got = ctx.bootstrap_wo_ks(ctx.to_device(cts))[:, :1025].cpu().numpy().view(np.uint32)
     finally:
         ctx.set_br_variant(6)
+        ctx.set_narrow_lanes(148)
     for k in range(9):
         assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), k
 
@@ -162,6 +174,7 @@ def test_mux_and_not(tb, ctx, keys):
 def test_lanes_per_cta_and_ragged_tail(tb, ctx, keys, lanes):
     """5 gates over CTAs of 1..4 lanes (ragged last CTA); stride 640 rows."""
     ctx.set_lanes_per_cta(lanes)
+    ctx.set_narrow_lanes(0)
     try:
         A, B = synth.random_bits(5, 40 + lanes), synth.random_bits(5, 50 + lanes)
         ca, cb = enc(keys, A, 60 + lanes), enc(keys, B, 70 + lanes)
@@ -169,6 +182,7 @@ def test_lanes_per_cta_and_ragged_tail(tb, ctx, keys, lanes):
         assert (out == O.gates(keys, O.XOR, ca, cb)).all()
     finally:
         ctx.set_lanes_per_cta(2)
+        ctx.set_narrow_lanes(148)
 
 
 def test_edge_cases(tb, ctx, keys):
