@@ -206,6 +206,60 @@ def mnist_mlp_tile(n_in: int = 16, n_out: int = 2, bits: int = 8):
     return B.arrays(outs)
 
 
+def _relu(B: Builder, x):
+    """signed two's-complement x (LSB first, MSB = sign) -> max(x, 0) as unsigned bits[:-1]"""
+    s = x[-1]
+    return [B.gate(ANDNY, s, xi) for xi in x[:-1]]      # !sign & bit
+
+
+def _max(B: Builder, x, y):
+    lt = _less_than(B, x, y)
+    return [B.gate(MUX, lt, y[k], x[k]) for k in range(len(x))]
+
+
+def mnist_fig4(side: int = 26, bits: int = 8, n_out: int = 10, pool: int = 3):
+    """cfg 5: the ChiselTorch MNIST model of Fig. 4 on `side` x `side` encrypted signed `bits`-bit
+    activations: ReLU -> MaxPool2d(pool, 1) -> Flatten -> Linear(((side-pool+1)^2), n_out) with encrypted
+    unsigned `bits`-bit weights (array multipliers + adder tree).  Fig. 4 declares Float(8,8); BASELINE asks
+    for an 8-bit quantised network, so integers are used (SURVEY 8(d) cfg 5).  Inputs: activations (row-major,
+    LSB first), then weights [n_out][features].  The default size has ~2.2 M gates."""
+    n_act = side * side
+    feat_side = side - pool + 1
+    n_feat = feat_side * feat_side
+    B = Builder(n_act * bits + n_out * n_feat * (bits - 1))
+    act = [list(range(i * bits, (i + 1) * bits)) for i in range(n_act)]
+    r = [_relu(B, a) for a in act]                                   # bits-1 unsigned bits each
+    feats = []
+    for y in range(feat_side):
+        for x in range(feat_side):
+            win = [r[(y + dy) * side + (x + dx)] for dy in range(pool) for dx in range(pool)]
+            while len(win) > 1:                                      # max tree
+                nxt = [_max(B, win[k], win[k + 1]) for k in range(0, len(win) - 1, 2)]
+                if len(win) % 2:
+                    nxt.append(win[-1])
+                win = nxt
+            feats.append(win[0])
+    wb = bits - 1
+    base = n_act * bits
+    outs = []
+    for o in range(n_out):
+        prods = []
+        for i in range(n_feat):
+            w = list(range(base + (o * n_feat + i) * wb, base + (o * n_feat + i + 1) * wb))
+            rows = [[B.gate(AND, feats[i][k], w[j]) for k in range(len(feats[i]))] for j in range(wb)]
+            acc = rows[0]
+            for j in range(1, wb):
+                acc = acc[:j] + _add(B, acc[j:], rows[j])
+            prods.append(acc)
+        while len(prods) > 1:
+            nxt = [_add(B, prods[k], prods[k + 1]) for k in range(0, len(prods) - 1, 2)]
+            if len(prods) % 2:
+                nxt.append(prods[-1])
+            prods = nxt
+        outs += prods[0]
+    return B.arrays(outs)
+
+
 def pack_bits(values, bits: int) -> np.ndarray:
     """unsigned ints -> LSB-first bit array"""
     v = np.asarray(values, np.uint64)

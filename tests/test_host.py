@@ -204,6 +204,27 @@ def test_mnist_tile_dot_products():
     assert (got == np.einsum("bi,boi->bo", act, W)).all()
 
 
+def test_mnist_fig4_network_computes_relu_maxpool_linear():
+    n = synth.mnist_fig4(side=5, bits=4, n_out=2, pool=3)
+    rng = np.random.default_rng(4)
+    for _ in range(4):
+        act, W = rng.integers(-8, 8, 25), rng.integers(0, 8, (2, 9))
+        x = np.concatenate([synth.pack_bits(act & 15, 4), synth.pack_bits(W.reshape(-1), 3)])
+        out = _eval(n, x[None])[0]
+        r = np.maximum(act, 0).reshape(5, 5)
+        f = np.array([r[y:y + 3, c:c + 3].max() for y in range(3) for c in range(3)])
+        assert synth.unpack_bits(out, len(out) // 2).tolist() == (W @ f).tolist()
+
+
+def test_mnist_fig4_full_size_shape(tb):
+    """SURVEY 8(d) cfg 5: ~2 M gates, ~130 levels, >90 % of gates in levels >= 8192 wide"""
+    n = synth.mnist_fig4()
+    lv, nl = tb.Netlist(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"]).levels()
+    w = np.bincount(lv)[1:]
+    assert 1_500_000 < len(n["type"]) < 3_000_000 and 100 < nl < 160
+    assert w[w >= 8192].sum() / w.sum() > 0.9
+
+
 def test_independent_level_shape():
     n = synth.independent_level(64, 5)
     assert n["n_inputs"] == 128 and set(np.unique(n["type"]).tolist()) <= {6, 7}
