@@ -43,6 +43,8 @@ void launch_bk_to_ntt(const uint32_t* bk, uint32_t* bkhat, const uint2* twF, uin
 void launch_build_gate_desc(int kind, int32_t wa, int32_t wb, uint32_t cst, int64_t count, LaneDesc* lanes,
                             GateDesc* gates, cudaStream_t st);
 int launch_ks(const KsArgs& A, int tile, cudaStream_t st);
+int launch_ks_split(const KsArgs& A, uint32_t* partial, cudaStream_t st);   // narrow levels
+size_t ks_split_scratch_words(int64_t ngates);
 void launch_ksk_relayout(const uint32_t* src, uint32_t* dst, cudaStream_t st);
 int set_ntt_constants(const uint32_t* fw, const uint32_t* fwp, const uint32_t* iw, const uint32_t* iwp,
                       const uint32_t* misc);

@@ -94,6 +94,86 @@ __global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A) {
     }
 }
 
+// ---- narrow levels: one gate's key switch split over S CTAs ---------------------------------------
+// A level with few gates leaves the tiled kernel with a handful of CTAs that each walk all 8,192 (i, j) digit
+// groups one after another.  Here CTA (g, s) owns input coefficients i in slice s of [0, N) for gate g and writes
+// its partial sum (words mod 2^32) to scratch; ks_reduce_kernel adds the S partials (integer sums mod 2^32 are
+// order-independent, so the result is bit-identical to the tiled kernel).
+constexpr int kKsSplit = 16;
+
+__global__ void __launch_bounds__(kKsThreads) ks_split_kernel(KsArgs A, uint32_t* __restrict__ partial) {
+    constexpr int I = kN / kKsSplit;
+    __shared__ uint16_t sW[I];
+    __shared__ uint32_t sB;
+    const int tid = threadIdx.x, gi = blockIdx.x, s = blockIdx.y;
+    const GateDesc gd = A.gates[gi];
+    const bool boot = gd.kind != kGateNot;
+    const uint32_t* l0 = A.lanes + (int64_t)(gd.lane0 - A.lane_base) * A.lane_stride;
+    const uint32_t* l1 = gd.lane1 >= 0 ? A.lanes + (int64_t)(gd.lane1 - A.lane_base) * A.lane_stride : nullptr;
+    for (int ii = tid; ii < I; ii += kKsThreads) {
+        uint32_t e = 0u;
+        if (boot) {
+            e = __ldg(l0 + s * I + ii);
+            if (l1) e += __ldg(l1 + s * I + ii);
+        }
+        sW[ii] = boot ? (uint16_t)((e + (1u << 15)) >> 16) : (uint16_t)0;
+    }
+    if (tid == 0) {
+        uint32_t b = 0u;
+        if (boot) {
+            b = __ldg(l0 + kN);
+            if (l1) b += __ldg(l1 + kN) + kMu;
+        }
+        sB = b;
+    }
+    __syncthreads();
+    const int k0 = 4 * tid;
+    if (k0 >= kKsRow) return;
+    uint32_t acc[4];
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+        const int k = k0 + q;
+        uint32_t v = 0u;
+        if (s == 0) {
+            if (!boot && k <= kn) v = 0u - __ldg(A.not_src + (int64_t)gd.lane0 * A.not_stride + k);
+            else if (k == kn) v = sB;
+        }
+        acc[q] = v;
+    }
+    for (int ii = 0; ii < I; ii++) {
+        const uint32_t w = sW[ii];
+        const uint32_t* rowi = A.ksk + (size_t)(s * I + ii) * kKsT * (kKsBase - 1) * kKsRow + k0;
+#pragma unroll
+        for (int j = 0; j < kKsT; j++) {
+            const uint32_t d = (w >> (14 - 2 * j)) & 3u;
+            if (d) {
+                const uint4 v = __ldg(reinterpret_cast<const uint4*>(rowi + (j * (kKsBase - 1) + d - 1) * kKsRow));
+                acc[0] -= v.x; acc[1] -= v.y; acc[2] -= v.z; acc[3] -= v.w;
+            }
+        }
+    }
+    *reinterpret_cast<uint4*>(partial + ((size_t)gi * kKsSplit + s) * kKsRow + k0) = make_uint4(acc[0], acc[1], acc[2], acc[3]);
+}
+
+__global__ void __launch_bounds__(kKsThreads) ks_reduce_kernel(KsArgs A, const uint32_t* __restrict__ partial) {
+    const int gi = blockIdx.x;
+    uint32_t* o = A.out + (int64_t)A.gates[gi].out_row * A.out_stride;
+    for (int k = threadIdx.x; k <= kn; k += kKsThreads) {
+        uint32_t v = 0u;
+#pragma unroll
+        for (int s = 0; s < kKsSplit; s++) v += partial[((size_t)gi * kKsSplit + s) * kKsRow + k];
+        o[k] = v;
+    }
+}
+
+int launch_ks_split(const KsArgs& A, uint32_t* partial, cudaStream_t st) {
+    if (A.ngates <= 0) return 0;
+    ks_split_kernel<<<dim3(A.ngates, kKsSplit), kKsThreads, 0, st>>>(A, partial);
+    ks_reduce_kernel<<<A.ngates, kKsThreads, 0, st>>>(A, partial);
+    return 0;
+}
+size_t ks_split_scratch_words(int64_t ngates) { return (size_t)ngates * kKsSplit * kKsRow; }
+
 // digit-0 rows dropped, rows padded to 632 words: [i][j][d][631] (host layout) -> [i][j][d-1][632]
 __global__ void ksk_relayout_kernel(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst) {
     const size_t row = blockIdx.x;                   // (i, j, d-1)

@@ -81,6 +81,8 @@ struct tb_ctx {
     size_t hwires_words = 0;
     int64_t* hidx = nullptr;                // tb_run_netlist_host gather rows
     int64_t hidx_n = 0;
+    uint32_t* ks_scratch = nullptr;         // split key-switch partial sums (narrow levels)
+    size_t ks_scratch_words = 0;
     // per-kernel event timing (tb_profile_*)
     bool prof = false;
     std::vector<cudaEvent_t> ev_pool;
@@ -230,6 +232,7 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
     cudaFree(c->stage);
     cudaFree(c->hwires);
     cudaFree(c->hidx);
+    cudaFree(c->ks_scratch);
     for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
     if (c->own) cudaStreamDestroy(c->own);
     delete c;
@@ -367,9 +370,22 @@ static int run_ks(tb_ctx* c, const uint32_t* lanes, int64_t lane_base, int64_t l
     A.lanes = lanes; A.lane_base = (int32_t)lane_base; A.lane_stride = lane_stride; A.gates = gates;
     A.ngates = (int32_t)ngates; A.ksk = c->ksk; A.out = out; A.out_stride = ostride; A.not_src = not_src;
     A.not_stride = not_stride;
+    const bool split = c->narrow_lanes > 0 && ngates <= c->narrow_lanes;   // narrow level: split each gate's KS
+    if (split && c->ks_scratch_words < ks_split_scratch_words(ngates)) {
+        cudaFree(c->ks_scratch);
+        c->ks_scratch = nullptr;
+        c->ks_scratch_words = 0;
+        const size_t words = ks_split_scratch_words(std::max<int64_t>(ngates, c->narrow_lanes));
+        if (cudaMalloc(&c->ks_scratch, words * 4) != cudaSuccess) {
+            cudaGetLastError();
+            return fail(TB_ENOMEM, "key-switch scratch allocation failed");
+        }
+        c->ks_scratch_words = words;
+    }
     const long slot = prof_begin(c, 1, st);
-    if (launch_ks(A, c->ks_tile, st)) return fail(TB_ECUDA, "key-switch kernel attribute/launch failed");
+    const int rc = split ? launch_ks_split(A, c->ks_scratch, st) : launch_ks(A, c->ks_tile, st);
     prof_end(c, slot, st);
+    if (rc) return fail(TB_ECUDA, "key-switch kernel attribute/launch failed");
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "ks_kernel launch");
     return TB_OK;

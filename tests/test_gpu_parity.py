@@ -127,13 +127,19 @@ def test_structured_key_closed_form(tb):
 
 
 # ------------------------------------------------------------------------------------- key switch
-def test_keyswitch_bit_exact(tb, ctx, keys):
+@pytest.mark.parametrize("narrow", [148, 0])
+def test_keyswitch_bit_exact(tb, ctx, keys, narrow):
+    """split key switch (narrow levels, 16 CTAs per gate) and tiled key switch (ragged: 4 tiles of 8 + 5)"""
     rng = np.random.default_rng(6)
-    ext = rng.integers(0, M32, (37, 1025), dtype=np.uint64).astype(np.uint32)    # ragged: 2 tiles + 5
+    ext = rng.integers(0, M32, (37, 1025), dtype=np.uint64).astype(np.uint32)
     ext[0, :] = 0
     ext[1, :1024] = 0xFFFFFFFF
     dev = ctx.to_device(ext, stride=1028)
-    got = ctx.to_host(ctx.keyswitch(dev))
+    ctx.set_narrow_lanes(narrow)
+    try:
+        got = ctx.to_host(ctx.keyswitch(dev))
+    finally:
+        ctx.set_narrow_lanes(148)
     for r in range(ext.shape[0]):
         assert (got[r] == O.keyswitch(keys, ext[r])).all(), r
 
