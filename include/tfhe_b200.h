@@ -167,6 +167,10 @@ int tb_set_br_variant(tb_ctx* ctx, int variant);
 /* Latency mode for narrow levels: a launch with <= `lanes` bootstraps uses br7 with one lane per CTA (one
  * SM per bootstrap, BK step staged in shared memory).  Default = the device's SM count; 0 disables. */
 int tb_set_narrow_lanes(tb_ctx* ctx, int64_t lanes);
+/* Latency-mode kernel: 9 = br9_kernel (default; one bootstrap per cluster of 2 SMs, each SM owning one
+ * accumulator polynomial, forward-NTT rows exchanged through distributed shared memory), 7 = br7<1> (one
+ * bootstrap per SM).  Bit-identical. */
+int tb_set_narrow_kernel(tb_ctx* ctx, int kernel);
 /* Gates per key-switch CTA (8, 16 or 32; default 8): each tile streams the 62 MB KSK once from L2. */
 int tb_set_ks_tile(tb_ctx* ctx, int gates);
 /* Device bytes a context holds for keys (BK NTT + KSK). */

@@ -126,6 +126,10 @@ class Context:
         """levels with <= lanes bootstraps run in latency mode (br7, one lane per SM); 0 disables"""
         _native.check(_native.lib().tb_set_narrow_lanes(self._h, lanes))
 
+    def set_narrow_kernel(self, kernel: int):
+        """latency-mode kernel: 9 = br9 (2-SM cluster per bootstrap, default), 7 = br7<1> (one SM)"""
+        _native.check(_native.lib().tb_set_narrow_kernel(self._h, kernel))
+
     def set_ks_tile(self, gates: int):
         """gates per key-switch CTA: 8 (default), 16 or 32"""
         _native.check(_native.lib().tb_set_ks_tile(self._h, gates))

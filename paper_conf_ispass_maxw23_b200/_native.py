@@ -90,6 +90,7 @@ SIGNATURES = {
     "tb_set_br_variant": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_set_ks_tile": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_set_narrow_lanes": (ctypes.c_int, [_vp, _i64]),
+    "tb_set_narrow_kernel": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_key_bytes": (ctypes.c_int, [_vp, ctypes.POINTER(_sz)]),
     "tb_microbench": (ctypes.c_int, [_vp, ctypes.c_int, ctypes.POINTER(ctypes.c_double),
                                      ctypes.POINTER(ctypes.c_double)]),

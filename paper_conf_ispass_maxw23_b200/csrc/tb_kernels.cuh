@@ -38,6 +38,7 @@ struct KsArgs {
 int launch_br6(const BrArgs& A, int G, cudaStream_t st);
 int launch_br7(const BrArgs& A, int G, cudaStream_t st);
 int launch_br8(const BrArgs& A, cudaStream_t st);
+int launch_br9(const BrArgs& A, cudaStream_t st);
 void launch_bk_to_ntt(const uint32_t* bk, uint32_t* bkhat, const uint2* twF, uint32_t ninv, uint32_t ninvp,
                       cudaStream_t st);
 void launch_build_gate_desc(int kind, int32_t wa, int32_t wb, uint32_t cst, int64_t count, LaneDesc* lanes,

@@ -3,6 +3,7 @@
 #include "tb_br6.cu"
 #include "tb_br7.cu"
 #include "tb_br8.cu"
+#include "tb_br9.cu"
 #include "tb_keyswitch.cu"
 #include "tb_diag.cu"
 #include "tb_runtime.cu"

@@ -61,7 +61,8 @@ struct tb_ctx {
     int lanes_per_cta = 2;
     int variant = 6;                        // blind-rotation kernel: 6 = br6, 7 = br7 (TMA-staged BK), 8 = br8
     int ks_tile = 8;                        // gates per key-switch CTA (8, 16, 32); 8 measured fastest
-    int narrow_lanes = 0;                   // levels with <= this many lanes use br7<1> (set to the SM count)
+    int narrow_lanes = 0;                   // launches with <= this many lanes run in latency mode (= SM count)
+    int narrow_kernel = 9;                  // latency-mode kernel: 9 = br9 (2-SM cluster per lane), 7 = br7<1>
     cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
     uint2* twF = nullptr;                   // [31][32]
     uint2* twI = nullptr;
@@ -251,6 +252,12 @@ extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
     return TB_OK;
 }
 
+extern "C" int tb_set_narrow_kernel(tb_ctx* c, int kernel) {
+    if (!c || (kernel != 7 && kernel != 9)) return fail(TB_EINVAL, "latency-mode kernel must be 7 or 9");
+    c->narrow_kernel = kernel;
+    return TB_OK;
+}
+
 extern "C" int tb_set_narrow_lanes(tb_ctx* c, int64_t lanes) {
     if (!c || lanes < 0) return fail(TB_EINVAL, "narrow-level threshold must be >= 0");
     c->narrow_lanes = lanes;
@@ -349,7 +356,8 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     const long slot = prof_begin(c, 0, st);
     int rc;
     if (c->narrow_lanes > 0 && nlanes <= c->narrow_lanes)
-        rc = launch_br7(A, 1, st);                      // narrow level: one lane per SM, BK staged per step
+        rc = c->narrow_kernel == 9 ? launch_br9(A, st)   // narrow level: one lane per 2-SM cluster
+                                   : launch_br7(A, 1, st);  // or one lane per SM, BK staged per step
     else if (c->variant == 7)
         rc = launch_br7(A, 2, st);
     else if (c->variant == 8)
