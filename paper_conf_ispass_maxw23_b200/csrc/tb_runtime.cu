@@ -403,7 +403,7 @@ extern "C" int tb_gates(tb_ctx* c, int gate, const uint32_t* ca, const uint32_t*
                         uint32_t* out, int64_t count, int64_t stride, tb_stream stream) {
     int rc = check_ready(c);
     if (rc) return rc;
-    if (count < 0 || stride < kn + 1 || count > (int64_t)1 << 30) return fail(TB_EINVAL, "bad count or stride");
+    if (count < 0 || stride < kn + 1 || count > ((int64_t)1 << 29)) return fail(TB_EINVAL, "bad count or stride");
     if (!gate_known(gate)) return fail(TB_EINVAL, "unknown gate code");
     if (count == 0) return TB_OK;
     if (!ca || !out || (gate != TB_NOT && !cb) || (gate == TB_MUX && !cc)) return fail(TB_EINVAL, "null array");

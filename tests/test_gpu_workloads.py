@@ -120,3 +120,46 @@ def test_run_netlist_host_matches_device(tb, ctx, keys):
     ref, dnet = run(tb, ctx, n, cts)
     out = ctx.run_netlist_host(dnet, cts, n["outputs"])
     assert (out == ref[n["outputs"]]).all()
+    rev = n["outputs"][::-1].copy()                              # non-contiguous rows -> device gather path
+    assert (ctx.run_netlist_host(dnet, cts, rev) == ref[rev]).all()
+    wide = np.zeros((cts.shape[0], 700), np.uint32)              # host input rows with a wider stride
+    wide[:, :631] = cts
+    assert (ctx.run_netlist_host(dnet, wide, np.array([0, n["n_inputs"]])) == ref[[0, n["n_inputs"]]]).all()
+
+
+def test_same_wire_twice_and_duplicate_consumers(tb, ctx, keys):
+    """XOR(a, a) = 0 and AND(a, a) = a; one wire feeding many gates of a level"""
+    n = dict(n_inputs=2, type=np.array([6, 8, 7, 7, 14], np.int32), in0=np.array([0, 0, 0, 1, 2]),
+             in1=np.array([0, 0, 1, 0, 3]), in2=np.full(5, -1), outputs=np.arange(2, 7))
+    bits = np.array([1, 0], np.uint8)
+    cts = O.encrypt_bits(keys, bits, 14)
+    w, _ = run(tb, ctx, n, cts)
+    ref = run_oracle_levels(keys, n, cts)
+    assert (w == ref).all()
+    assert O.decrypt_bits(keys, w[2:]).tolist() == [0, 1, 1, 1, 1]
+
+
+def run_oracle_levels(keys, n, cts):
+    from oracle.algorithm1 import algorithm1
+    w = np.zeros((n["n_inputs"] + len(n["type"]), 631), np.uint32)
+    w[:n["n_inputs"]] = cts
+    for batch in algorithm1(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"]):
+        b = np.array(batch)
+        O.run_level(keys, w, n["type"][b], n["in0"][b], n["in1"][b], n["in2"][b], n["n_inputs"] + b)
+    return w
+
+
+def test_errors_without_keys_and_bad_arguments(tb):
+    import torch
+    c = tb.Context(0)
+    x = c.empty(2)
+    with pytest.raises(tb.TBError) as e:
+        c.gates(tb.NAND, x, x)
+    assert e.value.code == -3                                     # TB_ENOKEYS
+    with pytest.raises(tb.TBError):
+        c.set_br_variant(5)
+    with pytest.raises(tb.TBError):
+        c.set_ks_tile(12)
+    with pytest.raises(ValueError):
+        c.gates(tb.NAND, x, x[:, :600])                           # shape mismatch caught in the binding
+    c.close()
