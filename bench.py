@@ -156,7 +156,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--gates-per-gpu", type=int, default=65536)
     ap.add_argument("--lanes-per-cta", type=int, default=2)
-    ap.add_argument("--br-variant", type=int, default=6, choices=[6, 7, 8])
+    ap.add_argument("--br-variant", type=int, default=6, choices=[6, 7, 8, 10])
     ap.add_argument("--ks-tile", type=int, default=8, choices=[8, 16, 32])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")

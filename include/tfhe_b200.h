@@ -157,10 +157,14 @@ int tb_keyswitch(tb_ctx* ctx, const uint32_t* in, int64_t in_stride, uint32_t* o
  * (digits[r] (x) polys[r])[c] mod 2^32, digits in [-64, 63], polys u32 torus.  All DEVICE pointers:
  * digits [6][N] int32, polys [6][N] u32, res [N] u32.  Synchronous. */
 int tb_ntt_muladd6(tb_ctx* ctx, const int32_t* digits, const uint32_t* polys, uint32_t* res);
+/* Same product through the FP64-pipe transform (folded 512-point complex negacyclic FFT, 16-bit signed BK
+ * halves, rounding to the nearest integer).  Synchronous. */
+int tb_fft_muladd6(tb_ctx* ctx, const int32_t* digits, const uint32_t* polys, uint32_t* res);
 
 /* Blind-rotation lanes per CTA for the default kernel (1..4, default 2); tuning knob. */
 int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
-/* Blind-rotation kernel: 6 = br6_kernel (default: 6 warps/lane, 2 CTAs/SM, BK words from L2), 7 = br7_kernel
+/* Blind-rotation kernel: 6 = br6_kernel (default: 6 warps/lane, 2 CTAs/SM, BK words from L2), 8 = br8_kernel
+ * (two ping-ponged lane groups per CTA), 10 = brf_kernel (FP64-pipe FFT), 7 = br7_kernel
  * (2 lanes/CTA, 1 CTA/SM, each 144 KB BK step TMA-bulk-copied into shared memory one step ahead).  Both are
  * bit-identical; see DESIGN.md "Kernels". */
 int tb_set_br_variant(tb_ctx* ctx, int variant);

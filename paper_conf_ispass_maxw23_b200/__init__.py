@@ -194,6 +194,12 @@ class Context:
                                                    _ptr(res)))
         return res
 
+    def fft_muladd6(self, digits: torch.Tensor, polys: torch.Tensor) -> torch.Tensor:
+        res = torch.empty(N_RING, dtype=torch.int32, device=self.device)
+        _native.check(_native.lib().tb_fft_muladd6(self._h, _ptr(digits.contiguous()), _ptr(polys.contiguous()),
+                                                   _ptr(res)))
+        return res
+
     def microbench(self, iters: int = 4096):
         b, m = ctypes.c_double(), ctypes.c_double()
         _native.check(_native.lib().tb_microbench(self._h, iters, ctypes.byref(b), ctypes.byref(m)))

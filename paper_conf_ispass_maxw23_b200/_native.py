@@ -86,6 +86,7 @@ SIGNATURES = {
     "tb_bootstrap_wo_ks": (ctypes.c_int, [_vp, _vp, _i64, _vp, _i64, _i64, _vp]),
     "tb_keyswitch": (ctypes.c_int, [_vp, _vp, _i64, _vp, _i64, _i64, _vp]),
     "tb_ntt_muladd6": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
+    "tb_fft_muladd6": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
     "tb_set_lanes_per_cta": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_set_br_variant": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_set_ks_tile": (ctypes.c_int, [_vp, ctypes.c_int]),

@@ -1,0 +1,234 @@
+// tb_brf.cu -- blind rotation on the FP64 pipe.
+//
+// Same CMux as br6 (bit-identical output), with the exact negacyclic products computed by the folded
+// 512-point complex transform of tb_fft.cuh instead of the integer NTT: the integer kernels are bound by the
+// IMAD pipe, and B200 executes DFMA at the IMAD rate on a separate pipe.  Each torus BK coefficient is split
+// into two signed 16-bit halves (x = lo + 2^16 hi mod 2^32); per output polynomial q the two half products
+// are exact integers of magnitude < 2^33.6, recovered by rounding, and recombined mod 2^32.
+// Per CMux step and lane (6 warps):
+//   A  warp r = bloc*3 + jd: digit jd of (X^abar - 1) ACC[bloc], folded, forward transform -> slot r
+//   B  thread item (position k, lane g): out[o][k] = sum_r D_r[k] * BKf_i[r][o][k] for the 4 outputs
+//      o = (q, half), complex FMA, written back in place (slots 0..3)
+//   C  warp o < 4: inverse transform, unfold, round, (<< 16 for the high half); the two half warps of q meet
+//      at a named barrier and the low-half warp adds both into ACC[q]
+#include "tb_fft.cuh"
+#include "tb_kernels.cuh"
+
+namespace tb {
+
+constexpr int kFOuts = 4;                       // (q, half)
+constexpr int kFStepD2 = kRows * kFOuts * 512;  // double2 per CMux step = 196,608 B
+
+template <int G>
+struct BrfSmem {
+    double2 twB[15 * 32];
+    double2 twC[8 * 32];
+    double2 slot[G][kRows][512];
+    uint32_t acc[G][2][kN];
+    uint16_t bar[G][kn + 2];
+};
+
+__device__ __forceinline__ double small_to_double(uint32_t v, double bias) {   // v < 2^31 exactly, minus bias
+    return __hiloint2double(0x43300000, (int)v) - (4503599627370496.0 + bias);
+}
+
+template <int G>
+__global__ void __launch_bounds__(192 * G, 1) brf_kernel(BrArgs A, const double2* __restrict__ bkf,
+                                                          const double2* __restrict__ twB,
+                                                          const double2* __restrict__ twC) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    BrfSmem<G>& S = *reinterpret_cast<BrfSmem<G>*>(smem_raw);
+    constexpr int NT = 192 * G;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int g = warp / 6, w6 = warp % 6;
+    const int lane0 = blockIdx.x * G;
+
+    for (int k = tid; k < 15 * 32; k += NT) S.twB[k] = twB[k];
+    for (int k = tid; k < 8 * 32; k += NT) S.twC[k] = twC[k];
+    {   // a1, a2
+        const int gl = lane0 + g;
+        LaneDesc d = {0, -1, 0, 0, 0u, 0u, 0u, 0u};
+        if (gl < A.nlanes) d = A.lanes[gl];
+        const uint32_t sa = d.sel & 3u, sb = (d.sel >> 2) & 3u;
+        const uint32_t* s0 = sa == 0 ? A.src0 : (sa == 1 ? A.src1 : A.src2);
+        const uint32_t* s1 = sb == 0 ? A.src0 : (sb == 1 ? A.src1 : A.src2);
+        const uint32_t* pa = s0 + (int64_t)d.ia * A.src_stride;
+        const uint32_t* pb = d.ib >= 0 ? s1 + (int64_t)d.ib * A.src_stride : nullptr;
+        for (int w = w6 * 32 + lane; w <= kn; w += 192) {
+            uint32_t v = (gl < A.nlanes) ? (uint32_t)d.wa * __ldg(pa + w) : 0u;
+            if (pb) v += (uint32_t)d.wb * __ldg(pb + w);
+            if (w == kn) v += d.cst;
+            S.bar[g][w] = (uint16_t)((v + (1u << 20)) >> 21);
+        }
+    }
+    __syncthreads();
+    for (int k = tid; k < G * kN; k += NT) {                  // a3
+        const int gg = k / kN, c = k % kN;
+        const uint32_t bbar = S.bar[gg][kn];
+        S.acc[gg][0][c] = 0u;
+        S.acc[gg][1][c] = ((c + bbar) & (kTwoN - 1)) < (uint32_t)kN ? kMu : (uint32_t)(0u - kMu);
+    }
+    __syncthreads();
+
+    const int bloc = w6 / kL, jd = w6 % kL;
+    const int q = w6 >> 1, h = w6 & 1;                        // phase C role (w6 < 4)
+    const int shift = 32 - kBgbit * (jd + 1);
+    for (int i = 0; i < kn; i++) {
+        {   // ---- A ----
+            const uint32_t ab = S.bar[g][i];
+            const uint32_t* acc = S.acc[g][bloc];
+            dcplx x[16];
+#pragma unroll
+            for (int j = 0; j < 16; j++) {
+                double v2[2];
+#pragma unroll
+                for (int half = 0; half < 2; half++) {
+                    const uint32_t c = lane + 32 * j + 512 * half;
+                    const uint32_t mm = (c - ab) & (kTwoN - 1);
+                    const uint32_t src = acc[mm & (kN - 1)];
+                    const uint32_t rot = mm < (uint32_t)kN ? src : 0u - src;
+                    const uint32_t u = rot - acc[c] + kDecompOffset;
+                    v2[half] = small_to_double((u >> shift) & 127u, 64.0);   // digit in [-64, 63]
+                }
+                x[j] = dcplx{v2[0], v2[1]};                                    // fold: a_k + i a_{k+512}
+            }
+            double2* slot = S.slot[g][w6];
+            fft_fwd(x, slot, S.twB, S.twC, lane);
+            __syncwarp();
+#pragma unroll
+            for (int j = 0; j < 16; j++) slot[fswz(lay_c(lane, j))] = make_double2(x[j].re, x[j].im);
+        }
+        __syncthreads();
+        {   // ---- B ----
+            const double2* bki = bkf + (size_t)i * kFStepD2;
+            for (int it = tid; it < G * 512; it += NT) {
+                const int gg = it / 512, k = it % 512;
+                const int sk = fswz(k);
+                dcplx D[kRows];
+#pragma unroll
+                for (int r = 0; r < kRows; r++) {
+                    const double2 v = S.slot[gg][r][sk];
+                    D[r] = dcplx{v.x, v.y};
+                }
+#pragma unroll
+                for (int o = 0; o < kFOuts; o++) {
+                    double re = 0.0, im = 0.0;
+#pragma unroll
+                    for (int r = 0; r < kRows; r++) {
+                        const double2 b = __ldg(bki + (r * kFOuts + o) * 512 + k);
+                        re = fma(D[r].re, b.x, fma(-D[r].im, b.y, re));
+                        im = fma(D[r].re, b.y, fma(D[r].im, b.x, im));
+                    }
+                    S.slot[gg][o][sk] = make_double2(re, im);
+                }
+            }
+        }
+        __syncthreads();
+        if (w6 < kFOuts) {   // ---- C ----
+            double2* slot = S.slot[g][w6];
+            dcplx x[16];
+#pragma unroll
+            for (int j = 0; j < 16; j++) {
+                const double2 v = slot[fswz(lay_c(lane, j))];
+                x[j] = dcplx{v.x, v.y};
+            }
+            fft_inv(x, slot, S.twB, S.twC, lane);
+            uint32_t v[32];
+#pragma unroll
+            for (int j = 0; j < 16; j++) {
+                v[j] = round_mod32(x[j].re) << (16 * h);                  // coefficient lane + 32 j
+                v[j + 16] = round_mod32(x[j].im) << (16 * h);             // coefficient lane + 32 j + 512
+            }
+            uint32_t* scratch = reinterpret_cast<uint32_t*>(slot);
+            __syncwarp();
+            if (h == 1) {
+#pragma unroll
+                for (int j = 0; j < 32; j++) scratch[lane + 32 * j] = v[j];
+            }
+            asm volatile("bar.sync %0, 64;" ::"r"(1 + g * 2 + q) : "memory");
+            if (h == 0) {
+                const uint32_t* other = reinterpret_cast<const uint32_t*>(S.slot[g][w6 + 1]);
+                uint32_t* accq = S.acc[g][q];
+#pragma unroll
+                for (int j = 0; j < 32; j++) accq[lane + 32 * j] += v[j] + other[lane + 32 * j];
+            }
+        }
+        __syncthreads();
+    }
+    {   // a5
+        const int gl = lane0 + g;
+        if (gl < A.nlanes) {
+            uint32_t* o = A.out + (int64_t)gl * A.out_stride;
+            for (int j = w6 * 32 + lane; j <= kN; j += 192) {
+                uint32_t v;
+                if (j == 0) v = S.acc[g][0][0];
+                else if (j < kN) v = 0u - S.acc[g][0][kN - j];
+                else v = S.acc[g][1][0];
+                o[j] = v;
+            }
+        }
+    }
+}
+
+// BK (torus) -> FFT domain: one warp per (i, r, q, half); stored [i][r][o = q*2 + half][k], scaled by 1/512
+__global__ void __launch_bounds__(128) bk_to_fft_kernel(const uint32_t* __restrict__ bk, double2* __restrict__ bkf,
+                                                        const double2* twB, const double2* twC) {
+    __shared__ double2 buf[4][512];
+    __shared__ double2 tB[15 * 32], tC[8 * 32];
+    for (int k = threadIdx.x; k < 15 * 32; k += blockDim.x) tB[k] = twB[k];
+    for (int k = threadIdx.x; k < 8 * 32; k += blockDim.x) tC[k] = twC[k];
+    __syncthreads();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int task = blockIdx.x * 4 + warp;
+    if (task >= kn * kRows * 2 * 2) return;
+    const int half = task & 1, q = (task >> 1) & 1, r = (task >> 2) % kRows, i = (task >> 2) / kRows;
+    const uint32_t* src = bk + (((size_t)i * kRows + r) * 2 + q) * kN;
+    dcplx x[16];
+#pragma unroll
+    for (int j = 0; j < 16; j++) {
+        double v[2];
+#pragma unroll
+        for (int f = 0; f < 2; f++) {
+            const uint32_t w = src[lane + 32 * j + 512 * f];
+            const int32_t lo = (int32_t)(int16_t)(w & 0xFFFFu);
+            const int32_t hi = (int32_t)(int16_t)((w - (uint32_t)lo) >> 16);
+            v[f] = (double)(half == 0 ? lo : hi);
+        }
+        x[j] = dcplx{v[0], v[1]};
+    }
+    fft_fwd(x, buf[warp], tB, tC, lane);
+    double2* dst = bkf + ((size_t)i * kRows + r) * kFOuts * 512 + (q * 2 + half) * 512;
+#pragma unroll
+    for (int j = 0; j < 16; j++) dst[lay_c(lane, j)] = make_double2(x[j].re * (1.0 / 512), x[j].im * (1.0 / 512));
+}
+
+template <int G>
+static int launch_brf_g(const BrArgs& A, const double2* bkf, const double2* twB, const double2* twC, cudaStream_t st) {
+    const size_t smem = sizeof(BrfSmem<G>);
+    static bool attr = false;
+    if (!attr) {
+        if (cudaFuncSetAttribute(brf_kernel<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+            return -1;
+        attr = true;
+    }
+    const int blocks = (A.nlanes + G - 1) / G;
+    if (blocks == 0) return 0;
+    brf_kernel<G><<<blocks, 192 * G, smem, st>>>(A, bkf, twB, twC);
+    return 0;
+}
+
+int launch_brf(const BrArgs& A, int G, const double2* bkf, const double2* twB, const double2* twC, cudaStream_t st) {
+    switch (G) {
+        case 1: return launch_brf_g<1>(A, bkf, twB, twC, st);
+        case 2: return launch_brf_g<2>(A, bkf, twB, twC, st);
+        default: return launch_brf_g<3>(A, bkf, twB, twC, st);
+    }
+}
+
+void launch_bk_to_fft(const uint32_t* bk, double2* bkf, const double2* twB, const double2* twC, cudaStream_t st) {
+    const int tasks = kn * kRows * 2 * 2;
+    bk_to_fft_kernel<<<(tasks + 3) / 4, 128, 0, st>>>(bk, bkf, twB, twC);
+}
+size_t bkf_bytes() { return (size_t)kn * kFStepD2 * sizeof(double2); }
+
+}  // namespace tb

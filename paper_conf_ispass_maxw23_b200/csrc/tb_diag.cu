@@ -176,3 +176,112 @@ int run_microbench(int iters, double* bfly, double* mac) {
 }
 
 }  // namespace tb
+
+// ---- FP64 FFT variant: diagnostic exact product (same transforms as the FFT blind-rotation kernel) ------
+#include "tb_fft.cuh"
+
+namespace tb {
+
+int set_fft_constants(const double2* zeta16) {
+    return cudaMemcpyToSymbol(c_zeta, zeta16, 16 * sizeof(double2)) == cudaSuccess ? 0 : -1;
+}
+
+// signed 16-bit halves of a torus word: x = lo + 2^16 hi (mod 2^32), lo, hi in [-2^15, 2^15)
+__device__ __forceinline__ void split16(uint32_t x, int32_t& lo, int32_t& hi) {
+    lo = (int32_t)(int16_t)(x & 0xFFFFu);
+    hi = (int32_t)(int16_t)((x - (uint32_t)lo) >> 16);
+}
+
+struct FftDiagSmem {
+    double2 twB[15 * 32];
+    double2 twC[8 * 32];
+    double2 d[kRows][512];
+    double2 b[kRows][2][512];
+};
+
+__global__ void __launch_bounds__(192) fft_muladd6_kernel(const int32_t* digits, const uint32_t* polys, uint32_t* res,
+                                                          const double2* twB, const double2* twC) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    FftDiagSmem& S = *reinterpret_cast<FftDiagSmem*>(smem_raw);
+    const int lane = threadIdx.x & 31, r = threadIdx.x >> 5;
+    for (int k = threadIdx.x; k < 15 * 32; k += blockDim.x) S.twB[k] = twB[k];
+    for (int k = threadIdx.x; k < 8 * 32; k += blockDim.x) S.twC[k] = twC[k];
+    __syncthreads();
+    dcplx x[16];
+#pragma unroll
+    for (int j = 0; j < 16; j++) {
+        const int k = lay_a(lane, j);
+        x[j] = dcplx{(double)digits[r * kN + k], (double)digits[r * kN + k + 512]};
+    }
+    fft_fwd(x, S.d[r], S.twB, S.twC, lane);
+    __syncwarp();
+#pragma unroll
+    for (int j = 0; j < 16; j++) S.d[r][fswz(lay_c(lane, j))] = make_double2(x[j].re, x[j].im);
+    for (int h = 0; h < 2; h++) {
+#pragma unroll
+        for (int j = 0; j < 16; j++) {
+            const int k = lay_a(lane, j);
+            int32_t l0, h0, l1, h1;
+            split16(polys[r * kN + k], l0, h0);
+            split16(polys[r * kN + k + 512], l1, h1);
+            x[j] = h == 0 ? dcplx{(double)l0, (double)l1} : dcplx{(double)h0, (double)h1};
+        }
+        fft_fwd(x, S.b[r][h], S.twB, S.twC, lane);
+        __syncwarp();
+#pragma unroll
+        for (int j = 0; j < 16; j++)
+            S.b[r][h][fswz(lay_c(lane, j))] = make_double2(x[j].re * (1.0 / 512), x[j].im * (1.0 / 512));
+    }
+    __syncthreads();
+    // MAC into d[0] (h = 0) and d[1] (h = 1): thread owns positions k
+    for (int k = threadIdx.x; k < 512; k += blockDim.x) {
+        const int sk = fswz(k);
+        dcplx D[kRows];
+#pragma unroll
+        for (int rr = 0; rr < kRows; rr++) D[rr] = dcplx{S.d[rr][sk].x, S.d[rr][sk].y};
+#pragma unroll
+        for (int h = 0; h < 2; h++) {
+            dcplx acc = {0.0, 0.0};
+#pragma unroll
+            for (int rr = 0; rr < kRows; rr++) {
+                const dcplx B = {S.b[rr][h][sk].x, S.b[rr][h][sk].y};
+                acc.re = fma(D[rr].re, B.re, fma(-D[rr].im, B.im, acc.re));
+                acc.im = fma(D[rr].re, B.im, fma(D[rr].im, B.re, acc.im));
+            }
+            S.d[h][sk] = make_double2(acc.re, acc.im);
+        }
+    }
+    __syncthreads();
+    if (r < 2) {
+#pragma unroll
+        for (int j = 0; j < 16; j++) {
+            const double2 v = S.d[r][fswz(lay_c(lane, j))];
+            x[j] = dcplx{v.x, v.y};
+        }
+        fft_inv(x, S.d[r], S.twB, S.twC, lane);
+        __syncwarp();
+        uint32_t* part = reinterpret_cast<uint32_t*>(S.b[r][0]);   // 1024 u32 scratch per half
+#pragma unroll
+        for (int j = 0; j < 16; j++) {
+            const int k = lay_a(lane, j);
+            part[k] = round_mod32(x[j].re);
+            part[k + 512] = round_mod32(x[j].im);
+        }
+    }
+    __syncthreads();
+    const uint32_t* lo = reinterpret_cast<const uint32_t*>(S.b[0][0]);
+    const uint32_t* hi = reinterpret_cast<const uint32_t*>(S.b[1][0]);
+    for (int c = threadIdx.x; c < kN; c += blockDim.x) res[c] = lo[c] + (hi[c] << 16);
+}
+
+int launch_fft_muladd6(const int32_t* digits, const uint32_t* polys, uint32_t* res, const double2* twB,
+                       const double2* twC, cudaStream_t st) {
+    const size_t smem = sizeof(FftDiagSmem);
+    if (cudaFuncSetAttribute(fft_muladd6_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+        cudaSuccess)
+        return -1;
+    fft_muladd6_kernel<<<1, 192, smem, st>>>(digits, polys, res, twB, twC);
+    return 0;
+}
+
+}  // namespace tb

@@ -1,0 +1,164 @@
+// tb_fft.cuh -- warp-level negacyclic transform of length 1024 in double precision, on the FP64 pipe (sm_100a).
+//
+// Alternative engine for the exact products of the CMux: a real polynomial
+// a mod X^1024 + 1 is folded to z = a mod (X^512 - i), z_k = a_k + i a_{k+512}, and transformed by stages 1..9
+// of the merged-twist Cooley-Tukey tree of X^1024 + 1 (zeta_{s,b} = psi^brv10(2^s + b), psi = e^{i pi/1024}),
+// i.e. evaluated at the 512 roots of X^512 = i.  Pointwise products + the Gentleman-Sande inverse + unfold give
+// the negacyclic product.  With 16-bit signed BK halves every product coefficient is an integer of magnitude
+// <= 6 * 1024 * 64 * 2^15 = 2^33.6 and the rounding error of the whole pipeline is < 1e-3, so rounding to the
+// nearest integer recovers it exactly.
+//
+// One warp owns one transform, 16 complex values per lane, three register layouts (k = transform index):
+//   A: k = t + 32 j            stages 1-4 in-thread, warp-uniform twiddles (constant bank)
+//   B: k = 32 (t>>1) + 2 j + (t&1)   stages 5-8 in-thread, per-lane twiddles (shared table, 15 per lane)
+//   C: k = 16 t + j            stage 9 in-thread, per-lane twiddles (8 per lane)
+// Transposes go through a 512 x 16-B shared buffer whose 16-B granules are XOR-swizzled so that all six access
+// patterns are bank-conflict free.
+#pragma once
+#include "tb_common.cuh"
+
+namespace tb {
+
+// stages 1-4 twiddles: index (2^(s-1) - 1) + b for s = 1..4 (15 entries), as (re, im)
+__constant__ double2 c_zeta[16];
+
+struct dcplx {
+    double re, im;
+};
+
+__device__ __forceinline__ int fswz(int k) {   // swizzled 16-B slot of transform index k
+    return (k & ~7) | ((k ^ ((k >> 4) & 1) ^ (((k >> 5) & 3) << 1)) & 7);
+}
+__device__ __forceinline__ int lay_a(int t, int j) { return t + 32 * j; }
+__device__ __forceinline__ int lay_b(int t, int j) { return ((t >> 1) << 5) | (j << 1) | (t & 1); }
+__device__ __forceinline__ int lay_c(int t, int j) { return (t << 4) | j; }
+
+__device__ __forceinline__ dcplx cmul(dcplx w, dcplx y) {
+    dcplx r;
+    r.re = fma(w.re, y.re, -w.im * y.im);
+    r.im = fma(w.re, y.im, w.im * y.re);
+    return r;
+}
+__device__ __forceinline__ dcplx cmulc(dcplx w, dcplx y) {   // conj(w) * y
+    dcplx r;
+    r.re = fma(w.re, y.re, w.im * y.im);
+    r.im = fma(w.re, y.im, -w.im * y.re);
+    return r;
+}
+__device__ __forceinline__ void ct_c(dcplx& x, dcplx& y, dcplx w) {
+    const dcplx t = cmul(w, y);
+    y.re = x.re - t.re;
+    y.im = x.im - t.im;
+    x.re += t.re;
+    x.im += t.im;
+}
+__device__ __forceinline__ void gs_c(dcplx& x, dcplx& y, dcplx w) {
+    const dcplx d = {x.re - y.re, x.im - y.im};
+    x.re += y.re;
+    x.im += y.im;
+    y = cmulc(w, d);
+}
+__device__ __forceinline__ dcplx ld_tw(const double2* t, int idx) {
+    const double2 v = t[idx];
+    return dcplx{v.x, v.y};
+}
+
+// One stage on 16 in-thread values: blocks of 2*LJ, NB blocks, twiddle of block bj from (a) the constant bank
+// (layout A: index CB + bj) or (b) a per-lane shared table (index (TB + bj) * 32 + lane).  Explicit template
+// instantiation keeps every register index a compile-time constant.
+template <int LJ, int NB, int CB>
+__device__ __forceinline__ void ct_stage_const(dcplx (&x)[16]) {
+#pragma unroll
+    for (int bj = 0; bj < NB; bj++) {
+        const double2 z = c_zeta[CB + bj];
+        const dcplx w = {z.x, z.y};
+#pragma unroll
+        for (int u = 0; u < LJ; u++) ct_c(x[bj * 2 * LJ + u], x[bj * 2 * LJ + u + LJ], w);
+    }
+}
+template <int LJ, int NB, int CB>
+__device__ __forceinline__ void gs_stage_const(dcplx (&x)[16]) {
+#pragma unroll
+    for (int bj = 0; bj < NB; bj++) {
+        const double2 z = c_zeta[CB + bj];
+        const dcplx w = {z.x, z.y};
+#pragma unroll
+        for (int u = 0; u < LJ; u++) gs_c(x[bj * 2 * LJ + u], x[bj * 2 * LJ + u + LJ], w);
+    }
+}
+template <int LJ, int NB, int TB>
+__device__ __forceinline__ void ct_stage_tab(dcplx (&x)[16], const double2* tw, int lane) {
+#pragma unroll
+    for (int bj = 0; bj < NB; bj++) {
+        const dcplx w = ld_tw(tw, (TB + bj) * 32 + lane);
+#pragma unroll
+        for (int u = 0; u < LJ; u++) ct_c(x[bj * 2 * LJ + u], x[bj * 2 * LJ + u + LJ], w);
+    }
+}
+template <int LJ, int NB, int TB>
+__device__ __forceinline__ void gs_stage_tab(dcplx (&x)[16], const double2* tw, int lane) {
+#pragma unroll
+    for (int bj = 0; bj < NB; bj++) {
+        const dcplx w = ld_tw(tw, (TB + bj) * 32 + lane);
+#pragma unroll
+        for (int u = 0; u < LJ; u++) gs_c(x[bj * 2 * LJ + u], x[bj * 2 * LJ + u + LJ], w);
+    }
+}
+
+// 16 values through the transpose buffer: write at layout FROM, read at layout TO (0 = A, 1 = B, 2 = C)
+template <int FROM, int TO>
+__device__ __forceinline__ void fft_transpose(dcplx (&x)[16], double2* buf, int lane) {
+    __syncwarp();
+#pragma unroll
+    for (int j = 0; j < 16; j++) {
+        const int k = FROM == 0 ? lay_a(lane, j) : (FROM == 1 ? lay_b(lane, j) : lay_c(lane, j));
+        buf[fswz(k)] = make_double2(x[j].re, x[j].im);
+    }
+    __syncwarp();
+#pragma unroll
+    for (int j = 0; j < 16; j++) {
+        const int k = TO == 0 ? lay_a(lane, j) : (TO == 1 ? lay_b(lane, j) : lay_c(lane, j));
+        const double2 v = buf[fswz(k)];
+        x[j] = dcplx{v.x, v.y};
+    }
+}
+
+// buf: 512 x double2 (8 KB) warp-private; twB: [15][32] per-lane twiddles of stages 5-8; twC: [8][32] stage 9
+// In: x[j] = z[lay_a(lane, j)].  Out: x[j] = Z[lay_c(lane, j)] (bit-reversed-order transform positions).
+__device__ __forceinline__ void fft_fwd(dcplx (&x)[16], double2* buf, const double2* twB, const double2* twC,
+                                        int lane) {
+    ct_stage_const<8, 1, 0>(x);       // stage 1 (pairs k bit 8)
+    ct_stage_const<4, 2, 1>(x);       // stage 2
+    ct_stage_const<2, 4, 3>(x);       // stage 3
+    ct_stage_const<1, 8, 7>(x);       // stage 4
+    fft_transpose<0, 1>(x, buf, lane);
+    ct_stage_tab<8, 1, 0>(x, twB, lane);    // stage 5 (pairs k bit 4)
+    ct_stage_tab<4, 2, 1>(x, twB, lane);    // stage 6
+    ct_stage_tab<2, 4, 3>(x, twB, lane);    // stage 7
+    ct_stage_tab<1, 8, 7>(x, twB, lane);    // stage 8
+    fft_transpose<1, 2>(x, buf, lane);
+    ct_stage_tab<1, 8, 0>(x, twC, lane);    // stage 9 (pairs k bit 0)
+}
+
+// In: x[j] = Z[lay_c(lane, j)].  Out: x[j] = 512 z[lay_a(lane, j)] (the 1/512 is folded into the stored BK).
+__device__ __forceinline__ void fft_inv(dcplx (&x)[16], double2* buf, const double2* twB, const double2* twC,
+                                        int lane) {
+    gs_stage_tab<1, 8, 0>(x, twC, lane);    // stage 9
+    fft_transpose<2, 1>(x, buf, lane);
+    gs_stage_tab<1, 8, 7>(x, twB, lane);    // stage 8
+    gs_stage_tab<2, 4, 3>(x, twB, lane);    // stage 7
+    gs_stage_tab<4, 2, 1>(x, twB, lane);    // stage 6
+    gs_stage_tab<8, 1, 0>(x, twB, lane);    // stage 5
+    fft_transpose<1, 0>(x, buf, lane);
+    gs_stage_const<1, 8, 7>(x);       // stage 4
+    gs_stage_const<2, 4, 3>(x);       // stage 3
+    gs_stage_const<4, 2, 1>(x);       // stage 2
+    gs_stage_const<8, 1, 0>(x);       // stage 1
+}
+
+// exact integer value (|v| < 2^51) of a double that is within 0.5 of it, reduced mod 2^32
+__device__ __forceinline__ uint32_t round_mod32(double v) {
+    return (uint32_t)__double2loint(v + 6755399441055744.0);   // 1.5 * 2^52: mantissa holds v + 2^51
+}
+
+}  // namespace tb

@@ -59,3 +59,15 @@ namespace tb {
 void launch_gather_rows(const uint32_t* src, int64_t stride, const int64_t* rows, int64_t n, uint32_t* out,
                         cudaStream_t st);
 }  // namespace tb
+
+namespace tb {
+int set_fft_constants(const double2* zeta16);
+int launch_fft_muladd6(const int32_t* digits, const uint32_t* polys, uint32_t* res, const double2* twB,
+                       const double2* twC, cudaStream_t st);
+}  // namespace tb
+
+namespace tb {
+int launch_brf(const BrArgs& A, int G, const double2* bkf, const double2* twB, const double2* twC, cudaStream_t st);
+void launch_bk_to_fft(const uint32_t* bk, double2* bkf, const double2* twB, const double2* twC, cudaStream_t st);
+size_t bkf_bytes();
+}  // namespace tb

@@ -66,8 +66,11 @@ struct tb_ctx {
     cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
     uint2* twF = nullptr;                   // [31][32]
     uint2* twI = nullptr;
+    double2* fftB = nullptr;                // FP64 FFT per-lane twiddles: stages 5-8 [15][32], stage 9 [8][32]
+    double2* fftC = nullptr;
     uint32_t ninv = 0, ninvp = 0;
     uint32_t* bkhat = nullptr;              // [n][6][6][N]
+    double2* bkf = nullptr;                 // FP64 variant: [n][6][4][512] complex, scaled by 1/512
     uint32_t* ksk = nullptr;                // [N][t][3][632]
     bool have_bk = false, have_ksk = false;
     // scratch (grown on demand; growing synchronises the device)
@@ -203,11 +206,30 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
                 tf[e * 32 + t] = make_uint2(w, shoup_of(w));
                 ti[e * 32 + t] = make_uint2(wi, shoup_of(wi));
             }
+    // FP64 FFT variant: psi = e^{i pi / 1024}; zeta_{s,b} = psi^brv10(2^s + b) (tb_fft.cuh), from long double
+    std::vector<double2> zeta16(16), fb(15 * 32), fc(8 * 32);
+    auto cpsi = [](uint32_t e) {
+        const long double a = 3.14159265358979323846264338327950288L * (long double)e / 1024.0L;
+        return make_double2((double)cosl(a), (double)sinl(a));
+    };
+    for (int s = 1; s <= 4; s++)
+        for (int b = 0; b < (1 << (s - 1)); b++) zeta16[(1 << (s - 1)) - 1 + b] = cpsi(brv10((1u << s) + b));
+    for (int s = 5; s <= 8; s++)
+        for (int bj = 0; bj < (1 << (s - 5)); bj++)
+            for (int t = 0; t < 32; t++)
+                fb[((1 << (s - 5)) - 1 + bj) * 32 + t] = cpsi(brv10((1u << s) + (uint32_t)(t >> 1) * (1u << (s - 5)) + bj));
+    for (int bj = 0; bj < 8; bj++)
+        for (int t = 0; t < 32; t++) fc[bj * 32 + t] = cpsi(brv10(512u + (uint32_t)t * 8u + bj));
     c->ninv = powmod(kN, kP - 2);
     c->ninvp = shoup_of(c->ninv);
     int rc = set_ntt_constants(fw, fwp, iw, iwp, misc);
+    if (rc == 0) rc = set_fft_constants(zeta16.data());
     cudaError_t e = cudaSuccess;
-    if (rc == 0) e = cudaStreamCreateWithFlags(&c->own, cudaStreamNonBlocking);
+    if (rc == 0) e = cudaMalloc(&c->fftB, fb.size() * sizeof(double2));
+    if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->fftC, fc.size() * sizeof(double2));
+    if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->fftB, fb.data(), fb.size() * sizeof(double2), cudaMemcpyHostToDevice);
+    if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->fftC, fc.data(), fc.size() * sizeof(double2), cudaMemcpyHostToDevice);
+    if (rc == 0 && e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->own, cudaStreamNonBlocking);
     if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->twF, 31 * 32 * sizeof(uint2));
     if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->twI, 31 * 32 * sizeof(uint2));
     if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->twF, tf.data(), tf.size() * sizeof(uint2), cudaMemcpyHostToDevice);
@@ -225,7 +247,10 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
     cudaSetDevice(c->device);
     cudaFree(c->twF);
     cudaFree(c->twI);
+    cudaFree(c->fftB);
+    cudaFree(c->fftC);
     cudaFree(c->bkhat);
+    cudaFree(c->bkf);
     cudaFree(c->ksk);
     cudaFree(c->lanebuf);
     cudaFree(c->ldesc);
@@ -247,7 +272,8 @@ extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
 }
 
 extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
-    if (!c || variant < 6 || variant > 8) return fail(TB_EINVAL, "blind-rotation variant must be 6, 7 or 8");
+    if (!c || !(variant == 6 || variant == 7 || variant == 8 || variant == 10))
+        return fail(TB_EINVAL, "blind-rotation variant must be 6, 7, 8 or 10");
     c->variant = variant;
     return TB_OK;
 }
@@ -283,11 +309,13 @@ extern "C" int tb_load_bk(tb_ctx* c, const uint32_t* host_bk, size_t n_words) {
     if (n_words != want) return fail(TB_EINVAL, "bootstrapping key must have n*2l*2*N words");
     TB_CUDA(cudaSetDevice(c->device));
     if (!c->bkhat) TB_CUDA(cudaMalloc(&c->bkhat, (size_t)kn * kRows * kOuts * kN * 4));
+    if (!c->bkf) TB_CUDA(cudaMalloc(&c->bkf, bkf_bytes()));
     uint32_t* tmp = nullptr;
     TB_CUDA(cudaMalloc(&tmp, want * 4));
     cudaError_t e = cudaMemcpyAsync(tmp, host_bk, want * 4, cudaMemcpyHostToDevice, c->own);
     if (e == cudaSuccess) {
         launch_bk_to_ntt(tmp, c->bkhat, c->twF, c->ninv, c->ninvp, c->own);
+        launch_bk_to_fft(tmp, c->bkf, c->fftB, c->fftC, c->own);
         e = cudaGetLastError();
     }
     if (e == cudaSuccess) e = cudaStreamSynchronize(c->own);
@@ -360,6 +388,8 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
                                    : launch_br7(A, 1, st);  // or one lane per SM, BK staged per step
     else if (c->variant == 7)
         rc = launch_br7(A, 2, st);
+    else if (c->variant == 10)
+        rc = launch_brf(A, std::min(std::max(c->lanes_per_cta, 1), 3), c->bkf, c->fftB, c->fftC, st);
     else if (c->variant == 8)
         rc = launch_br8(A, st);
     else
@@ -486,6 +516,16 @@ extern "C" int tb_ntt_muladd6(tb_ctx* c, const int32_t* digits, const uint32_t* 
     TB_CUDA(cudaSetDevice(c->device));
     if (launch_ntt_muladd6(digits, polys, res, c->twF, c->twI, c->ninv, c->ninvp, c->own))
         return fail(TB_ECUDA, "ntt_muladd6 launch failed");
+    TB_CUDA(cudaGetLastError());
+    TB_CUDA(cudaStreamSynchronize(c->own));
+    return TB_OK;
+}
+
+extern "C" int tb_fft_muladd6(tb_ctx* c, const int32_t* digits, const uint32_t* polys, uint32_t* res) {
+    if (!c || !digits || !polys || !res) return fail(TB_EINVAL, "null argument");
+    TB_CUDA(cudaSetDevice(c->device));
+    if (launch_fft_muladd6(digits, polys, res, c->fftB, c->fftC, c->own))
+        return fail(TB_ECUDA, "fft_muladd6 launch failed");
     TB_CUDA(cudaGetLastError());
     TB_CUDA(cudaStreamSynchronize(c->own));
     return TB_OK;

@@ -60,6 +60,24 @@ def test_ntt_product_equals_schoolbook(tb, ctx):
         assert (got.cpu().numpy().view(np.uint32) == want).all()
 
 
+def test_fft_product_equals_schoolbook(tb, ctx):
+    """FP64-pipe folded FFT product (16-bit BK halves) rounds to the exact schoolbook result, incl. worst case"""
+    import torch
+    rng = np.random.default_rng(3)
+    cases = [(rng.integers(-64, 64, (6, 1024)), rng.integers(0, M32, (6, 1024), dtype=np.uint64)),
+             (np.full((6, 1024), -64), np.full((6, 1024), 0x80008000, np.uint64)),      # |halves| = 2^15
+             (np.full((6, 1024), 63), np.full((6, 1024), M32 - 1, np.uint64)),
+             (rng.choice([-64, 63], (6, 1024)), rng.choice([0x80008000, 0x7FFF7FFF], (6, 1024)).astype(np.uint64))]
+    for d, b in cases:
+        d32 = d.astype(np.int32)
+        b32 = b.astype(np.uint32)
+        want = np.zeros(1024, np.uint32)
+        for r in range(6):
+            want = O.negacyclic_muladd(d32[r], b32[r], want)
+        got = ctx.fft_muladd6(torch.from_numpy(d32).cuda(), torch.from_numpy(b32.view(np.int32)).cuda())
+        assert (got.cpu().numpy().view(np.uint32) == want).all()
+
+
 # ------------------------------------------------------------------------------------- blind rotation
 def test_bootstrap_wo_ks_bit_exact(tb, ctx, keys):
     rng = np.random.default_rng(2)
@@ -87,7 +105,7 @@ def test_narrow_level_latency_mode_bit_exact(tb, ctx, keys, kernel):
         ctx.set_narrow_kernel(9)
 
 
-@pytest.mark.parametrize("variant", [6, 7, 8])
+@pytest.mark.parametrize("variant", [6, 7, 8, 10])
 def test_blind_rotation_variants_bit_exact(tb, ctx, keys, variant):
     """every blind-rotation kernel variant (br6 / br7 TMA-staged / br8 ping-pong) on a ragged batch of 9"""
     rng = np.random.default_rng(40 + variant)
