@@ -5,10 +5,11 @@
 // IMAD pipe, and B200 executes DFMA at the IMAD rate on a separate pipe.  Each torus BK coefficient is split
 // into two signed 16-bit halves (x = lo + 2^16 hi mod 2^32); per output polynomial q the two half products
 // are exact integers of magnitude < 2^33.6, recovered by rounding, and recombined mod 2^32.
-// Per CMux step and lane (6 warps):
-//   A  warp r = bloc*3 + jd: digit jd of (X^abar - 1) ACC[bloc], folded, forward transform -> slot r
-//   B  thread item (position k, lane g): out[o][k] = sum_r D_r[k] * BKf_i[r][o][k] for the 4 outputs
-//      o = (q, half), complex FMA, written back in place (slots 0..3)
+// Per CMux step, G lanes per CTA, 8 warps per lane:
+//   A  warp r = bloc*3 + jd < 6: digit jd of (X^abar - 1) ACC[bloc], folded, forward transform -> slot r
+//   B  thread item = position k for all G lanes: out[g][o][k] = sum_r D_{g,r}[k] * BKf_i[r][o][k] for the 4
+//      outputs o = (q, half), complex FMA, written back in place (slots 0..3); each BK word is loaded once
+//      per CTA and used G times
 //   C  warp o < 4: inverse transform, unfold, round, (<< 16 for the high half); the two half warps of q meet
 //      at a named barrier and the low-half warp adds both into ACC[q]
 #include "tb_fft.cuh"
@@ -32,15 +33,19 @@ __device__ __forceinline__ double small_to_double(uint32_t v, double bias) {   /
     return __hiloint2double(0x43300000, (int)v) - (4503599627370496.0 + bias);
 }
 
+constexpr int kFWarps = 8;   // warps per lane: 6 forward transforms, 512 MAC positions / 256 threads, 4 inverse
+
+// The G lanes of the CTA move in lockstep and share every BK load in the MAC (measured: letting the lanes
+// drift apart with per-lane named barriers and per-lane BK loads is 6 % slower).
 template <int G>
-__global__ void __launch_bounds__(192 * G, 1) brf_kernel(BrArgs A, const double2* __restrict__ bkf,
-                                                          const double2* __restrict__ twB,
-                                                          const double2* __restrict__ twC) {
+__global__ void __launch_bounds__(256 * G, G == 1 ? 2 : 1) brf_kernel(BrArgs A, const double2* __restrict__ bkf,
+                                                                      const double2* __restrict__ twB,
+                                                                      const double2* __restrict__ twC) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     BrfSmem<G>& S = *reinterpret_cast<BrfSmem<G>*>(smem_raw);
-    constexpr int NT = 192 * G;
+    constexpr int NT = 256 * G;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int g = warp / 6, w6 = warp % 6;
+    const int g = warp / kFWarps, w8 = warp % kFWarps;
     const int lane0 = blockIdx.x * G;
 
     for (int k = tid; k < 15 * 32; k += NT) S.twB[k] = twB[k];
@@ -54,7 +59,7 @@ __global__ void __launch_bounds__(192 * G, 1) brf_kernel(BrArgs A, const double2
         const uint32_t* s1 = sb == 0 ? A.src0 : (sb == 1 ? A.src1 : A.src2);
         const uint32_t* pa = s0 + (int64_t)d.ia * A.src_stride;
         const uint32_t* pb = d.ib >= 0 ? s1 + (int64_t)d.ib * A.src_stride : nullptr;
-        for (int w = w6 * 32 + lane; w <= kn; w += 192) {
+        for (int w = w8 * 32 + lane; w <= kn; w += 256) {
             uint32_t v = (gl < A.nlanes) ? (uint32_t)d.wa * __ldg(pa + w) : 0u;
             if (pb) v += (uint32_t)d.wb * __ldg(pb + w);
             if (w == kn) v += d.cst;
@@ -70,11 +75,14 @@ __global__ void __launch_bounds__(192 * G, 1) brf_kernel(BrArgs A, const double2
     }
     __syncthreads();
 
-    const int bloc = w6 / kL, jd = w6 % kL;
-    const int q = w6 >> 1, h = w6 & 1;                        // phase C role (w6 < 4)
+    // phase A role ra < 6: rotating the two idle roles by 2 per lane spreads the 6G busy warps evenly over
+    // the 4 SM sub-partitions (warp w runs on sub-partition w % 4)
+    const int ra = (w8 + 2 * g) % kFWarps;
+    const int bloc = ra / kL, jd = ra % kL;
+    const int q = w8 >> 1, h = w8 & 1;                        // phase C role (w8 < 4)
     const int shift = 32 - kBgbit * (jd + 1);
     for (int i = 0; i < kn; i++) {
-        {   // ---- A ----
+        if (ra < kRows) {   // ---- A ----
             const uint32_t ab = S.bar[g][i];
             const uint32_t* acc = S.acc[g][bloc];
             dcplx x[16];
@@ -92,44 +100,51 @@ __global__ void __launch_bounds__(192 * G, 1) brf_kernel(BrArgs A, const double2
                 }
                 x[j] = dcplx{v2[0], v2[1]};                                    // fold: a_k + i a_{k+512}
             }
-            double2* slot = S.slot[g][w6];
+            double2* slot = S.slot[g][ra];
             fft_fwd(x, slot, S.twB, S.twC, lane);
             __syncwarp();
 #pragma unroll
-            for (int j = 0; j < 16; j++) slot[fswz(lay_c(lane, j))] = make_double2(x[j].re, x[j].im);
+            for (int j = 0; j < 16; j++) slot[fswz(lay_d(lane, j))] = make_double2(x[j].re, x[j].im);
         }
         __syncthreads();
-        {   // ---- B ----
+        {   // ---- B: one BK load serves the G lanes of the CTA ----
             const double2* bki = bkf + (size_t)i * kFStepD2;
-            for (int it = tid; it < G * 512; it += NT) {
-                const int gg = it / 512, k = it % 512;
+#pragma unroll 1
+            for (int k = tid; k < 512; k += NT) {
                 const int sk = fswz(k);
-                dcplx D[kRows];
+                dcplx D[G][kRows];
 #pragma unroll
-                for (int r = 0; r < kRows; r++) {
-                    const double2 v = S.slot[gg][r][sk];
-                    D[r] = dcplx{v.x, v.y};
-                }
-#pragma unroll
-                for (int o = 0; o < kFOuts; o++) {
-                    double re = 0.0, im = 0.0;
+                for (int gm = 0; gm < G; gm++)
 #pragma unroll
                     for (int r = 0; r < kRows; r++) {
-                        const double2 b = __ldg(bki + (r * kFOuts + o) * 512 + k);
-                        re = fma(D[r].re, b.x, fma(-D[r].im, b.y, re));
-                        im = fma(D[r].re, b.y, fma(D[r].im, b.x, im));
+                        const double2 v = S.slot[gm][r][sk];
+                        D[gm][r] = dcplx{v.x, v.y};
                     }
-                    S.slot[gg][o][sk] = make_double2(re, im);
+#pragma unroll
+                for (int o = 0; o < kFOuts; o++) {
+                    double2 b[kRows];
+#pragma unroll
+                    for (int r = 0; r < kRows; r++) b[r] = __ldg(bki + (r * kFOuts + o) * 512 + k);
+#pragma unroll
+                    for (int gm = 0; gm < G; gm++) {
+                        double re = 0.0, im = 0.0;
+#pragma unroll
+                        for (int r = 0; r < kRows; r++) {
+                            re = fma(D[gm][r].re, b[r].x, fma(-D[gm][r].im, b[r].y, re));
+                            im = fma(D[gm][r].re, b[r].y, fma(D[gm][r].im, b[r].x, im));
+                        }
+                        S.slot[gm][o][sk] = make_double2(re, im);
+                    }
                 }
             }
         }
         __syncthreads();
-        if (w6 < kFOuts) {   // ---- C ----
-            double2* slot = S.slot[g][w6];
+        if (w8 < kFOuts) {   // ---- C ----
+            double2* slot = S.slot[g][w8];
             dcplx x[16];
 #pragma unroll
             for (int j = 0; j < 16; j++) {
-                const double2 v = slot[fswz(lay_c(lane, j))];
+                const double2 v = slot[fswz(lay_d(lane, j))];
                 x[j] = dcplx{v.x, v.y};
             }
             fft_inv(x, slot, S.twB, S.twC, lane);
@@ -147,7 +162,7 @@ __global__ void __launch_bounds__(192 * G, 1) brf_kernel(BrArgs A, const double2
             }
             asm volatile("bar.sync %0, 64;" ::"r"(1 + g * 2 + q) : "memory");
             if (h == 0) {
-                const uint32_t* other = reinterpret_cast<const uint32_t*>(S.slot[g][w6 + 1]);
+                const uint32_t* other = reinterpret_cast<const uint32_t*>(S.slot[g][w8 + 1]);
                 uint32_t* accq = S.acc[g][q];
 #pragma unroll
                 for (int j = 0; j < 32; j++) accq[lane + 32 * j] += v[j] + other[lane + 32 * j];
@@ -159,7 +174,7 @@ __global__ void __launch_bounds__(192 * G, 1) brf_kernel(BrArgs A, const double2
         const int gl = lane0 + g;
         if (gl < A.nlanes) {
             uint32_t* o = A.out + (int64_t)gl * A.out_stride;
-            for (int j = w6 * 32 + lane; j <= kN; j += 192) {
+            for (int j = w8 * 32 + lane; j <= kN; j += 256) {
                 uint32_t v;
                 if (j == 0) v = S.acc[g][0][0];
                 else if (j < kN) v = 0u - S.acc[g][0][kN - j];
@@ -199,7 +214,7 @@ __global__ void __launch_bounds__(128) bk_to_fft_kernel(const uint32_t* __restri
     fft_fwd(x, buf[warp], tB, tC, lane);
     double2* dst = bkf + ((size_t)i * kRows + r) * kFOuts * 512 + (q * 2 + half) * 512;
 #pragma unroll
-    for (int j = 0; j < 16; j++) dst[lay_c(lane, j)] = make_double2(x[j].re * (1.0 / 512), x[j].im * (1.0 / 512));
+    for (int j = 0; j < 16; j++) dst[lay_d(lane, j)] = make_double2(x[j].re * (1.0 / 512), x[j].im * (1.0 / 512));
 }
 
 template <int G>
@@ -213,15 +228,14 @@ static int launch_brf_g(const BrArgs& A, const double2* bkf, const double2* twB,
     }
     const int blocks = (A.nlanes + G - 1) / G;
     if (blocks == 0) return 0;
-    brf_kernel<G><<<blocks, 192 * G, smem, st>>>(A, bkf, twB, twC);
+    brf_kernel<G><<<blocks, 256 * G, smem, st>>>(A, bkf, twB, twC);
     return 0;
 }
 
 int launch_brf(const BrArgs& A, int G, const double2* bkf, const double2* twB, const double2* twC, cudaStream_t st) {
     switch (G) {
         case 1: return launch_brf_g<1>(A, bkf, twB, twC, st);
-        case 2: return launch_brf_g<2>(A, bkf, twB, twC, st);
-        default: return launch_brf_g<3>(A, bkf, twB, twC, st);
+        default: return launch_brf_g<2>(A, bkf, twB, twC, st);
     }
 }
 

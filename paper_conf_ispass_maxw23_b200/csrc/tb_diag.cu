@@ -216,7 +216,7 @@ __global__ void __launch_bounds__(192) fft_muladd6_kernel(const int32_t* digits,
     fft_fwd(x, S.d[r], S.twB, S.twC, lane);
     __syncwarp();
 #pragma unroll
-    for (int j = 0; j < 16; j++) S.d[r][fswz(lay_c(lane, j))] = make_double2(x[j].re, x[j].im);
+    for (int j = 0; j < 16; j++) S.d[r][fswz(lay_d(lane, j))] = make_double2(x[j].re, x[j].im);
     for (int h = 0; h < 2; h++) {
 #pragma unroll
         for (int j = 0; j < 16; j++) {
@@ -230,7 +230,7 @@ __global__ void __launch_bounds__(192) fft_muladd6_kernel(const int32_t* digits,
         __syncwarp();
 #pragma unroll
         for (int j = 0; j < 16; j++)
-            S.b[r][h][fswz(lay_c(lane, j))] = make_double2(x[j].re * (1.0 / 512), x[j].im * (1.0 / 512));
+            S.b[r][h][fswz(lay_d(lane, j))] = make_double2(x[j].re * (1.0 / 512), x[j].im * (1.0 / 512));
     }
     __syncthreads();
     // MAC into d[0] (h = 0) and d[1] (h = 1): thread owns positions k
@@ -255,7 +255,7 @@ __global__ void __launch_bounds__(192) fft_muladd6_kernel(const int32_t* digits,
     if (r < 2) {
 #pragma unroll
         for (int j = 0; j < 16; j++) {
-            const double2 v = S.d[r][fswz(lay_c(lane, j))];
+            const double2 v = S.d[r][fswz(lay_d(lane, j))];
             x[j] = dcplx{v.x, v.y};
         }
         fft_inv(x, S.d[r], S.twB, S.twC, lane);

@@ -9,11 +9,12 @@
 // nearest integer recovers it exactly.
 //
 // One warp owns one transform, 16 complex values per lane, three register layouts (k = transform index):
-//   A: k = t + 32 j            stages 1-4 in-thread, warp-uniform twiddles (constant bank)
+//   A: k = t + 32 j                  stages 1-4 in-thread, warp-uniform twiddles (constant bank)
 //   B: k = 32 (t>>1) + 2 j + (t&1)   stages 5-8 in-thread, per-lane twiddles (shared table, 15 per lane)
-//   C: k = 16 t + j            stage 9 in-thread, per-lane twiddles (8 per lane)
-// Transposes go through a 512 x 16-B shared buffer whose 16-B granules are XOR-swizzled so that all six access
-// patterns are bank-conflict free.
+//   D: k = 16 t + 2 (j&7) + (j>>3)   stage 9 pairs lanes t, t^1: each lane sends 8 values with one shuffle
+//                                    each and computes 8 butterflies (per-lane twiddles, 8 per lane)
+// D is the frequency-domain layout every caller (BK, MAC) uses.  The A <-> B transpose goes through a 512 x 16-B
+// shared buffer whose 16-B granules are XOR-swizzled so that every access pattern is bank-conflict free.
 #pragma once
 #include "tb_common.cuh"
 
@@ -32,6 +33,7 @@ __device__ __forceinline__ int fswz(int k) {   // swizzled 16-B slot of transfor
 __device__ __forceinline__ int lay_a(int t, int j) { return t + 32 * j; }
 __device__ __forceinline__ int lay_b(int t, int j) { return ((t >> 1) << 5) | (j << 1) | (t & 1); }
 __device__ __forceinline__ int lay_c(int t, int j) { return (t << 4) | j; }
+__device__ __forceinline__ int lay_d(int t, int j) { return (t << 4) | ((j & 7) << 1) | (j >> 3); }
 
 __device__ __forceinline__ dcplx cmul(dcplx w, dcplx y) {
     dcplx r;
@@ -123,8 +125,38 @@ __device__ __forceinline__ void fft_transpose(dcplx (&x)[16], double2* buf, int 
     }
 }
 
+__device__ __forceinline__ dcplx sel(bool p, dcplx a, dcplx b) { return p ? a : b; }
+__device__ __forceinline__ dcplx shfl_x1(dcplx v) {
+    return dcplx{__shfl_xor_sync(0xffffffffu, v.re, 1), __shfl_xor_sync(0xffffffffu, v.im, 1)};
+}
+
+// stage 9 forward: B -> D.  Lane pair (t even, t odd) holds positions 2b, 2b+1 of block b = 16 (t>>1) + j in
+// x[j]; the even lane computes the butterflies j < 8, the odd lane j >= 8 (block b = 8 t + m, m < 8).
+__device__ __forceinline__ void stage9_fwd(dcplx (&x)[16], const double2* twC, int lane) {
+    const bool p = lane & 1;
+#pragma unroll
+    for (int m = 0; m < 8; m++) {
+        const dcplx r = shfl_x1(sel(p, x[m], x[m + 8]));
+        dcplx e = sel(p, r, x[m]), o = sel(p, x[m + 8], r);
+        ct_c(e, o, ld_tw(twC, m * 32 + lane));
+        x[m] = e;
+        x[m + 8] = o;
+    }
+}
+// stage 9 inverse: D -> B
+__device__ __forceinline__ void stage9_inv(dcplx (&x)[16], const double2* twC, int lane) {
+    const bool p = lane & 1;
+#pragma unroll
+    for (int m = 0; m < 8; m++) {
+        gs_c(x[m], x[m + 8], ld_tw(twC, m * 32 + lane));
+        const dcplx r = shfl_x1(sel(p, x[m], x[m + 8]));
+        if (p) x[m] = r;
+        else x[m + 8] = r;
+    }
+}
+
 // buf: 512 x double2 (8 KB) warp-private; twB: [15][32] per-lane twiddles of stages 5-8; twC: [8][32] stage 9
-// In: x[j] = z[lay_a(lane, j)].  Out: x[j] = Z[lay_c(lane, j)] (bit-reversed-order transform positions).
+// In: x[j] = z[lay_a(lane, j)].  Out: x[j] = Z[lay_d(lane, j)] (bit-reversed-order transform positions).
 __device__ __forceinline__ void fft_fwd(dcplx (&x)[16], double2* buf, const double2* twB, const double2* twC,
                                         int lane) {
     ct_stage_const<8, 1, 0>(x);       // stage 1 (pairs k bit 8)
@@ -136,15 +168,13 @@ __device__ __forceinline__ void fft_fwd(dcplx (&x)[16], double2* buf, const doub
     ct_stage_tab<4, 2, 1>(x, twB, lane);    // stage 6
     ct_stage_tab<2, 4, 3>(x, twB, lane);    // stage 7
     ct_stage_tab<1, 8, 7>(x, twB, lane);    // stage 8
-    fft_transpose<1, 2>(x, buf, lane);
-    ct_stage_tab<1, 8, 0>(x, twC, lane);    // stage 9 (pairs k bit 0)
+    stage9_fwd(x, twC, lane);               // stage 9 (pairs k bit 0)
 }
 
-// In: x[j] = Z[lay_c(lane, j)].  Out: x[j] = 512 z[lay_a(lane, j)] (the 1/512 is folded into the stored BK).
+// In: x[j] = Z[lay_d(lane, j)].  Out: x[j] = 512 z[lay_a(lane, j)] (the 1/512 is folded into the stored BK).
 __device__ __forceinline__ void fft_inv(dcplx (&x)[16], double2* buf, const double2* twB, const double2* twC,
                                         int lane) {
-    gs_stage_tab<1, 8, 0>(x, twC, lane);    // stage 9
-    fft_transpose<2, 1>(x, buf, lane);
+    stage9_inv(x, twC, lane);               // stage 9
     gs_stage_tab<1, 8, 7>(x, twB, lane);    // stage 8
     gs_stage_tab<2, 4, 3>(x, twB, lane);    // stage 7
     gs_stage_tab<4, 2, 1>(x, twB, lane);    // stage 6

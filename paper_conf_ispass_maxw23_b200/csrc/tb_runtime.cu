@@ -389,7 +389,7 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     else if (c->variant == 7)
         rc = launch_br7(A, 2, st);
     else if (c->variant == 10)
-        rc = launch_brf(A, std::min(std::max(c->lanes_per_cta, 1), 3), c->bkf, c->fftB, c->fftC, st);
+        rc = launch_brf(A, std::min(std::max(c->lanes_per_cta, 1), 2), c->bkf, c->fftB, c->fftC, st);
     else if (c->variant == 8)
         rc = launch_br8(A, st);
     else
