@@ -106,9 +106,10 @@ def lib():
     """Load the in-tree shared library (raises if it has not been built)."""
     global _lib
     if _lib is None:
-        if not os.path.exists(SO_PATH):
-            raise RuntimeError("libtfhe_b200.so is not built (run __graft_entry__.build()); there is no CPU fallback")
-        L = ctypes.CDLL(SO_PATH)
+        path = os.environ.get("TB_LIB", SO_PATH)     # A/B timing of alternative builds (scratch/ab.sh)
+        if not os.path.exists(path):
+            raise RuntimeError("%s is not built (run __graft_entry__.build()); there is no CPU fallback" % path)
+        L = ctypes.CDLL(path)
         for name, (res, args) in SIGNATURES.items():
             f = getattr(L, name)
             f.restype = res

@@ -193,8 +193,8 @@ __device__ __forceinline__ void split16(uint32_t x, int32_t& lo, int32_t& hi) {
 }
 
 struct FftDiagSmem {
-    double2 twB[15 * 32];
-    double2 twC[8 * 32];
+    double2 twB[kTwB];
+    double2 twC[kTwC];
     double2 d[kRows][512];
     double2 b[kRows][2][512];
 };
@@ -204,8 +204,8 @@ __global__ void __launch_bounds__(192) fft_muladd6_kernel(const int32_t* digits,
     extern __shared__ __align__(128) unsigned char smem_raw[];
     FftDiagSmem& S = *reinterpret_cast<FftDiagSmem*>(smem_raw);
     const int lane = threadIdx.x & 31, r = threadIdx.x >> 5;
-    for (int k = threadIdx.x; k < 15 * 32; k += blockDim.x) S.twB[k] = twB[k];
-    for (int k = threadIdx.x; k < 8 * 32; k += blockDim.x) S.twC[k] = twC[k];
+    for (int k = threadIdx.x; k < kTwB; k += blockDim.x) S.twB[k] = twB[k];
+    for (int k = threadIdx.x; k < kTwC; k += blockDim.x) S.twC[k] = twC[k];
     __syncthreads();
     dcplx x[16];
 #pragma unroll

@@ -207,7 +207,7 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
                 ti[e * 32 + t] = make_uint2(wi, shoup_of(wi));
             }
     // FP64 FFT variant: psi = e^{i pi / 1024}; zeta_{s,b} = psi^brv10(2^s + b) (tb_fft.cuh), from long double
-    std::vector<double2> zeta16(16), fb(15 * 32), fc(8 * 32);
+    std::vector<double2> zeta16(16), fb(kTwB), fc(kTwC);
     auto cpsi = [](uint32_t e) {
         const long double a = 3.14159265358979323846264338327950288L * (long double)e / 1024.0L;
         return make_double2((double)cosl(a), (double)sinl(a));
@@ -215,11 +215,8 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
     for (int s = 1; s <= 4; s++)
         for (int b = 0; b < (1 << (s - 1)); b++) zeta16[(1 << (s - 1)) - 1 + b] = cpsi(brv10((1u << s) + b));
     for (int s = 5; s <= 8; s++)
-        for (int bj = 0; bj < (1 << (s - 5)); bj++)
-            for (int t = 0; t < 32; t++)
-                fb[((1 << (s - 5)) - 1 + bj) * 32 + t] = cpsi(brv10((1u << s) + (uint32_t)(t >> 1) * (1u << (s - 5)) + bj));
-    for (int bj = 0; bj < 8; bj++)
-        for (int t = 0; t < 32; t++) fc[bj * 32 + t] = cpsi(brv10(512u + (uint32_t)t * 8u + bj));
+        for (int u = 0; u < 16; u++) fb[(s - 5) * 16 + u] = cpsi(brv10((1u << s) + (uint32_t)u * (1u << (s - 5))));
+    for (int t = 0; t < 32; t++) fc[t] = cpsi(brv10(512u + (uint32_t)t * 8u));
     c->ninv = powmod(kN, kP - 2);
     c->ninvp = shoup_of(c->ninv);
     int rc = set_ntt_constants(fw, fwp, iw, iwp, misc);
@@ -389,7 +386,7 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     else if (c->variant == 7)
         rc = launch_br7(A, 2, st);
     else if (c->variant == 10)
-        rc = launch_brf(A, std::min(std::max(c->lanes_per_cta, 1), 2), c->bkf, c->fftB, c->fftC, st);
+        rc = launch_brf(A, std::min(std::max(c->lanes_per_cta, 1), 3), c->bkf, c->fftB, c->fftC, st);
     else if (c->variant == 8)
         rc = launch_br8(A, st);
     else

@@ -215,6 +215,24 @@ def test_lanes_per_cta_and_ragged_tail(tb, ctx, keys, lanes):
         ctx.set_narrow_lanes(148)
 
 
+@pytest.mark.parametrize("lanes", [1, 2, 3])
+def test_fft_variant_lanes_per_cta(tb, ctx, keys, lanes):
+    """FP64 variant at 1, 2, 3 lanes per CTA (16, 16, 18 warps): 7 bootstraps, so every CTA size has a ragged tail"""
+    rng = np.random.default_rng(80 + lanes)
+    cts = rng.integers(0, M32, (7, 631), dtype=np.uint64).astype(np.uint32)
+    ctx.set_br_variant(10)
+    ctx.set_lanes_per_cta(lanes)
+    ctx.set_narrow_lanes(0)
+    try:
+        got = ctx.bootstrap_wo_ks(ctx.to_device(cts))[:, :1025].cpu().numpy().view(np.uint32)
+    finally:
+        ctx.set_br_variant(6)
+        ctx.set_lanes_per_cta(2)
+        ctx.set_narrow_lanes(148)
+    for k in range(7):
+        assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), k
+
+
 def test_edge_cases(tb, ctx, keys):
     import torch
     empty = ctx.empty(0)
