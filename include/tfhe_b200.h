@@ -168,12 +168,15 @@ int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
  * (2 lanes/CTA, 1 CTA/SM, each 144 KB BK step TMA-bulk-copied into shared memory one step ahead).  Both are
  * bit-identical; see DESIGN.md "Kernels". */
 int tb_set_br_variant(tb_ctx* ctx, int variant);
-/* Latency mode for narrow levels: a launch with <= `lanes` bootstraps uses br7 with one lane per CTA (one
- * SM per bootstrap, BK step staged in shared memory).  Default = the device's SM count; 0 disables. */
+/* Latency mode for narrow levels: a launch with <= `lanes` bootstraps runs a latency-mode kernel (below)
+ * instead of the throughput kernel.  Default = the device's SM count; 0 disables. */
 int tb_set_narrow_lanes(tb_ctx* ctx, int64_t lanes);
-/* Latency-mode kernel: 9 = br9_kernel (default; one bootstrap per cluster of 2 SMs, each SM owning one
- * accumulator polynomial, forward-NTT rows exchanged through distributed shared memory), 7 = br7<1> (one
- * bootstrap per SM).  Bit-identical. */
+/* Latency-mode kernel: 0 = auto (default: brl while the level's bootstraps fit in one wave of brl clusters,
+ * else br9), 11 = brl_kernel (one bootstrap per cluster of 4 SMs on the FP64 path: each SM owns one output
+ * polynomial and one 16-bit BK half, transforms split over warp pairs; 2.2 ms per level on B200),
+ * 9 = br9_kernel (one bootstrap per cluster of 2 SMs, each SM owning one accumulator polynomial, forward-NTT
+ * rows exchanged through distributed shared memory; 4.2 ms), 7 = br7<1> (one bootstrap per SM).  All are
+ * bit-identical.  Anything else: TB_EINVAL. */
 int tb_set_narrow_kernel(tb_ctx* ctx, int kernel);
 /* Gates per key-switch CTA (8, 16 or 32; default 8): each tile streams the 62 MB KSK once from L2. */
 int tb_set_ks_tile(tb_ctx* ctx, int gates);

@@ -29,9 +29,6 @@ struct BrfSmem {
     uint16_t bar[G][kn + 2];
 };
 
-__device__ __forceinline__ double small_to_double(uint32_t v, double bias) {   // v < 2^31 exactly, minus bias
-    return __hiloint2double(0x43300000, (int)v) - (4503599627370496.0 + bias);
-}
 
 // Warps per lane: W = 8 for G <= 2 (6 forward transforms, 4 inverse; 16 warps, 126 registers), W = 6 for G = 3
 // (18 warps: more transforms in flight per SM; the register file is split over the 4 sub-partitions, so 5 warps

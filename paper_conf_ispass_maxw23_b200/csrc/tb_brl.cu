@@ -1,0 +1,382 @@
+// tb_brl.cu -- latency-mode blind rotation on the FP64 pipe: one bootstrap per thread-block cluster of four SMs
+// (SURVEY 8(f) f4 "single-gate latency path ... split across a thread-block cluster").
+//
+// Same CMux and the same exact FFT-domain products as brf (tb_fft.cuh),
+// so the output is bit-identical to every other variant.  What changes is how one CMux step is spread out, to
+// shorten the serial chain of 630 steps that bounds a narrow netlist level:
+//   * CTA (q, h) of the cluster (rank 2q + h) owns output polynomial q and BK half h: it computes the 3 digit
+//     rows of ACC[q] (the two CTAs of a q compute them redundantly), sends them to CTA (1-q, h), runs the MAC
+//     for its one output o = 2q + h over all 6 rows, and one inverse transform; the two CTAs of a q swap their
+//     rounded halves and both add lo + 2^16 hi into their copy of ACC[q].
+//   * every transform is split over 2 warps (64 threads x 8 values) and done as three radix-8 passes (stages
+//     1-3, 4-6, 7-9 of the merged-twist tree), with one shared-memory exchange between passes; the pass-2/3
+//     twiddles of a thread stay in registers for the whole kernel.
+//   * BK_i's 48 KB for output o are TMA-staged two steps ahead; rows and halves move CTA-to-CTA with
+//     shared::cluster bulk copies that complete on the receiver's mbarrier (double-buffered by step parity,
+//     safe for the same reason as br9's hand-over: a CTA can only send for step i+2 after it has received the
+//     receiver's data of step i+1, which the receiver produced after consuming step i).
+#include "tb_fft.cuh"
+#include "tb_kernels.cuh"
+
+namespace tb {
+
+constexpr int kLThreads = 192;                 // 6 warps: 3 forward transforms x 2 warps; warps 0-1 invert
+
+struct __align__(128) BrlSmem {
+    double2 bk[2][kRows][512];                 // BK_i, rows 0..5 of output o = 2q + h, by step parity (96 KB)
+    double2 dslot[kL][512];                    // own forward rows (bloc q), swizzled positions
+    double2 rrows[2][kL][512];                 // rows of bloc 1-q from CTA (1-q, h), by step parity
+    double2 oslot[512];                        // MAC output, then the inverse's exchange buffer
+    uint32_t res[kN];                          // own rounded half of the product (sent to the sibling)
+    uint32_t rres[2][kN];                      // the sibling's half, by step parity
+    uint32_t acc[3 * kN];                      // ACC[q] as (acc, -acc, acc)
+    uint16_t bar[kn + 2];
+    unsigned long long mbar_bk[2], mbar_rows[2], mbar_res[2];
+};
+
+// swizzled slot of transform position k: each of the three pass groupings below touches 8 distinct 16-byte
+// bank groups per 8 consecutive threads (conflict-free)
+__device__ __forceinline__ int lsw(int k) { return k ^ ((k >> 3) & 7); }
+// position of element v of thread tt in the groupings of pass 1 (bits 8-6 in-thread), 2 (bits 5-3), 3 (bits 2-0)
+__device__ __forceinline__ int gp1(int tt, int v) { return (v << 6) | tt; }
+__device__ __forceinline__ int gp2(int tt, int v) { return ((tt >> 3) << 6) | (v << 3) | (tt & 7); }
+__device__ __forceinline__ int gp3(int tt, int v) { return (tt << 3) | v; }
+
+struct PassTw {
+    dcplx a, b, c;    // zeta_{s, b0}, zeta_{s+1, 2 b0}, zeta_{s+2, 4 b0} for the pass's stages s, s+1, s+2
+};
+// twiddle of the third stage of a pass, block 4 b0 + f: the bits of f land on exponent bits 9, 8 of brv10
+__device__ __forceinline__ dcplx tw_third(dcplx c, int f) {
+    constexpr double c4 = 0.70710678118654752440;
+    const dcplx w = (f >> 1) ? mul_k(c, c4, c4) : c;
+    return (f & 1) ? mul_i(w) : w;
+}
+// element v = (v2 v1 v0): first stage pairs v2, second v1 (block 2 b0 + v2), third v0 (block 4 b0 + 2 v2 + v1)
+__device__ __forceinline__ void pass_fwd(dcplx (&x)[8], const PassTw& t) {
+#pragma unroll
+    for (int u = 0; u < 4; u++) ct_c(x[u], x[u + 4], t.a);
+#pragma unroll
+    for (int e = 0; e < 2; e++) {
+        const dcplx w = e ? mul_i(t.b) : t.b;
+#pragma unroll
+        for (int u = 0; u < 2; u++) ct_c(x[4 * e + u], x[4 * e + u + 2], w);
+    }
+#pragma unroll
+    for (int f = 0; f < 4; f++) ct_c(x[2 * f], x[2 * f + 1], tw_third(t.c, f));
+}
+__device__ __forceinline__ void pass_inv(dcplx (&x)[8], const PassTw& t) {
+#pragma unroll
+    for (int f = 0; f < 4; f++) gs_c(x[2 * f], x[2 * f + 1], tw_third(t.c, f));
+#pragma unroll
+    for (int e = 0; e < 2; e++) {
+        const dcplx w = e ? mul_i(t.b) : t.b;
+#pragma unroll
+        for (int u = 0; u < 2; u++) gs_c(x[4 * e + u], x[4 * e + u + 2], w);
+    }
+#pragma unroll
+    for (int u = 0; u < 4; u++) gs_c(x[u], x[u + 4], t.a);
+}
+__device__ __forceinline__ void bar_pair(int id) { asm volatile("bar.sync %0, 64;" ::"r"(id) : "memory"); }
+__device__ __forceinline__ dcplx ldc(const double2* p) {
+    const double2 v = *p;
+    return dcplx{v.x, v.y};
+}
+__device__ __forceinline__ void stc(double2* p, dcplx v) { *p = make_double2(v.re, v.im); }
+
+// forward transform by a warp pair.  In: x[v] = z[gp1(tt, v)].  Out: Z[k] at buf[lsw(k)] (written by this pair;
+// each thread writes back exactly the positions it read, so one barrier per exchange suffices).
+__device__ __forceinline__ void fwd2w(dcplx (&x)[8], double2* buf, const PassTw& t1, const PassTw& t2,
+                                      const PassTw& t3, int tt, int id) {
+    pass_fwd(x, t1);
+#pragma unroll
+    for (int v = 0; v < 8; v++) stc(buf + lsw(gp1(tt, v)), x[v]);
+    bar_pair(id);
+#pragma unroll
+    for (int v = 0; v < 8; v++) x[v] = ldc(buf + lsw(gp2(tt, v)));
+    pass_fwd(x, t2);
+#pragma unroll
+    for (int v = 0; v < 8; v++) stc(buf + lsw(gp2(tt, v)), x[v]);
+    bar_pair(id);
+#pragma unroll
+    for (int v = 0; v < 8; v++) x[v] = ldc(buf + lsw(gp3(tt, v)));
+    pass_fwd(x, t3);
+#pragma unroll
+    for (int v = 0; v < 8; v++) stc(buf + lsw(gp3(tt, v)), x[v]);
+}
+// inverse by a warp pair.  In: Z[k] at buf[lsw(k)] (complete).  Out: x[v] = 512 z[gp1(tt, v)].
+__device__ __forceinline__ void inv2w(dcplx (&x)[8], double2* buf, const PassTw& t1, const PassTw& t2,
+                                      const PassTw& t3, int tt, int id) {
+#pragma unroll
+    for (int v = 0; v < 8; v++) x[v] = ldc(buf + lsw(gp3(tt, v)));
+    pass_inv(x, t3);
+#pragma unroll
+    for (int v = 0; v < 8; v++) stc(buf + lsw(gp3(tt, v)), x[v]);
+    bar_pair(id);
+#pragma unroll
+    for (int v = 0; v < 8; v++) x[v] = ldc(buf + lsw(gp2(tt, v)));
+    pass_inv(x, t2);
+#pragma unroll
+    for (int v = 0; v < 8; v++) stc(buf + lsw(gp2(tt, v)), x[v]);
+    bar_pair(id);
+#pragma unroll
+    for (int v = 0; v < 8; v++) x[v] = ldc(buf + lsw(gp1(tt, v)));
+    pass_inv(x, t1);
+}
+
+__device__ __forceinline__ uint32_t sm32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ uint32_t cl_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ uint32_t cl_map(uint32_t a, uint32_t rank) {
+    uint32_t out;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(out) : "r"(a), "r"(rank));
+    return out;
+}
+__device__ __forceinline__ void cl_sync() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void mb_init(unsigned long long* b) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(sm32(b)) : "memory");
+}
+__device__ __forceinline__ void mb_expect(unsigned long long* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sm32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mb_wait(unsigned long long* b, uint32_t parity) {
+    asm volatile(
+        "{\n .reg .pred p;\n WL_%=:\n mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n"
+        " @!p bra WL_%=;\n}\n" ::"r"(sm32(b)),
+        "r"(parity)
+        : "memory");
+}
+// local shared -> peer shared bulk copy completing on the peer's mbarrier
+__device__ __forceinline__ void push_peer(uint32_t dst, const void* src, uint32_t bytes, uint32_t mbar) {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    asm volatile(
+        "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+        "r"(sm32(src)), "r"(bytes), "r"(mbar)
+        : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+// BK_i rows 0..5 of output o -> bk[buf] (one thread)
+__device__ __forceinline__ void issue_bk_l(BrlSmem& S, const double2* bkf, int i, int o, int buf) {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    mb_expect(&S.mbar_bk[buf], kRows * 512 * 16);
+#pragma unroll
+    for (int r = 0; r < kRows; r++)
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                sm32(S.bk[buf][r])),
+            "l"(bkf + ((size_t)(i * kRows + r) * 4 + o) * 512), "r"(512 * 16), "r"(sm32(&S.mbar_bk[buf]))
+            : "memory");
+}
+
+// twL: [64][6] per-thread pass bases: (pass 2: zeta_{4,t>>3}, zeta_{5,2(t>>3)}, zeta_{6,4(t>>3)},
+//       pass 3: zeta_{7,t}, zeta_{8,2t}, zeta_{9,4t}); pass 1 bases come from the constant bank
+__global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
+    brl_kernel(BrArgs A, const double2* __restrict__ bkf, const double2* __restrict__ twL) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    BrlSmem& S = *reinterpret_cast<BrlSmem*>(smem_raw);
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t rank = cl_rank();
+    const int q = (int)(rank >> 1), h = (int)(rank & 1), o = 2 * q + h;
+    const int gl = blockIdx.x >> 2;                      // one lane (bootstrap) per cluster
+
+    if (tid == 0) {
+        for (int b = 0; b < 2; b++) {
+            mb_init(&S.mbar_bk[b]);
+            mb_init(&S.mbar_rows[b]);
+            mb_init(&S.mbar_res[b]);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        for (int b = 0; b < 2; b++) {                    // rows and halves of steps 0 and 1 may arrive any time
+            mb_expect(&S.mbar_rows[b], kL * 512 * 16);
+            mb_expect(&S.mbar_res[b], kN * 4);
+        }
+    }
+    __syncthreads();
+    if (tid == 0) {
+        issue_bk_l(S, bkf, 0, o, 0);
+        issue_bk_l(S, bkf, 1, o, 1);
+    }
+    {   // a1, a2 (every CTA of the cluster)
+        LaneDesc d = {0, -1, 0, 0, 0u, 0u, 0u, 0u};
+        if (gl < A.nlanes) d = A.lanes[gl];
+        const uint32_t sa = d.sel & 3u, sb = (d.sel >> 2) & 3u;
+        const uint32_t* s0 = sa == 0 ? A.src0 : (sa == 1 ? A.src1 : A.src2);
+        const uint32_t* s1 = sb == 0 ? A.src0 : (sb == 1 ? A.src1 : A.src2);
+        const uint32_t* pa = s0 + (int64_t)d.ia * A.src_stride;
+        const uint32_t* pb = d.ib >= 0 ? s1 + (int64_t)d.ib * A.src_stride : nullptr;
+        for (int w = tid; w <= kn; w += kLThreads) {
+            uint32_t v = (gl < A.nlanes) ? (uint32_t)d.wa * __ldg(pa + w) : 0u;
+            if (pb) v += (uint32_t)d.wb * __ldg(pb + w);
+            if (w == kn) v += d.cst;
+            S.bar[w] = (uint16_t)((v + (1u << 20)) >> 21);
+        }
+    }
+    __syncthreads();
+    for (int k = tid; k < kN; k += kLThreads) {           // a3: ACC[0] = 0, ACC[1] = X^{-bbar} (mu, ..., mu)
+        const uint32_t bbar = S.bar[kn];
+        const uint32_t v = q == 0 ? 0u : (((k + bbar) & (kTwoN - 1)) < (uint32_t)kN ? kMu : (uint32_t)(0u - kMu));
+        S.acc[k] = S.acc[k + 2 * kN] = v;
+        S.acc[k + kN] = 0u - v;
+    }
+    cl_sync();                                            // every mbarrier of the cluster is initialised and armed
+
+    const int tt = (warp & 1) * 32 + lane;               // thread index within its warp pair
+    const int jd = warp >> 1;                             // forward role: digit jd of bloc q (warps 0-5)
+    const int shift = 32 - kBgbit * (jd + 1);
+    PassTw t1, t2, t3;
+    t1.a = dcplx{c_zeta[0].x, c_zeta[0].y};
+    t1.b = dcplx{c_zeta[1].x, c_zeta[1].y};
+    t1.c = dcplx{c_zeta[3].x, c_zeta[3].y};
+    t2.a = ldc(twL + tt * 6 + 0);
+    t2.b = ldc(twL + tt * 6 + 1);
+    t2.c = ldc(twL + tt * 6 + 2);
+    t3.a = ldc(twL + tt * 6 + 3);
+    t3.b = ldc(twL + tt * 6 + 4);
+    t3.c = ldc(twL + tt * 6 + 5);
+    const uint32_t rows_dst = cl_map(sm32(&S.rrows[0][0][0]), rank ^ 2u);
+    const uint32_t rows_mb = cl_map(sm32(&S.mbar_rows[0]), rank ^ 2u);
+    const uint32_t res_dst = cl_map(sm32(&S.rres[0][0]), rank ^ 1u);
+    const uint32_t res_mb = cl_map(sm32(&S.mbar_res[0]), rank ^ 1u);
+
+    for (int i = 0; i < kn; i++) {
+        const int buf = i & 1;
+        const uint32_t par = (uint32_t)((i >> 1) & 1);
+        {   // ---- A: digit jd of (X^abar - 1) ACC[q], folded, forward transform (warp pair jd) ----
+            const uint32_t ab = S.bar[i];
+            const uint32_t* win = S.acc + ((tt - (int)ab) & (kTwoN - 1));
+            dcplx x[8];
+#pragma unroll
+            for (int v = 0; v < 8; v++) {
+                const int c = gp1(tt, v);
+                const uint32_t u0 = win[64 * v] - S.acc[c] + kDecompOffset;
+                const uint32_t u1 = win[64 * v + 512] - S.acc[c + 512] + kDecompOffset;
+                x[v] = dcplx{small_to_double((u0 >> shift) & 127u, 64.0), small_to_double((u1 >> shift) & 127u, 64.0)};
+            }
+            fwd2w(x, S.dslot[jd], t1, t2, t3, tt, 1 + jd);
+        }
+        __syncthreads();
+        if (tid == 0)   // our 3 rows -> CTA (1-q, h)
+            push_peer(rows_dst + (uint32_t)(buf * kL * 512 * 16), &S.dslot[0][0], kL * 512 * 16,
+                      rows_mb + (uint32_t)(buf * 8));
+        mb_wait(&S.mbar_bk[buf], par);
+        // ---- B: out[k] = sum_{r<6} D_r[k] BK_i[r][o][k]; own bloc's rows first, then the other bloc's ----
+        dcplx m3[3];
+#pragma unroll
+        for (int e = 0; e < 3; e++) {
+            const int k = tid + kLThreads * e;
+            dcplx s = {0.0, 0.0};
+            if (k < 512) {
+#pragma unroll
+                for (int r = 0; r < kL; r++) {
+                    const dcplx d = ldc(&S.dslot[r][lsw(k)]), b = ldc(&S.bk[buf][q * kL + r][k]);
+                    s.re = fma(d.re, b.re, fma(-d.im, b.im, s.re));
+                    s.im = fma(d.re, b.im, fma(d.im, b.re, s.im));
+                }
+            }
+            m3[e] = s;
+        }
+        mb_wait(&S.mbar_rows[buf], par);
+#pragma unroll
+        for (int e = 0; e < 3; e++) {
+            const int k = tid + kLThreads * e;
+            if (k < 512) {
+                dcplx s = m3[e];
+#pragma unroll
+                for (int r = 0; r < kL; r++) {
+                    const dcplx d = ldc(&S.rrows[buf][r][lsw(k)]), b = ldc(&S.bk[buf][(1 - q) * kL + r][k]);
+                    s.re = fma(d.re, b.re, fma(-d.im, b.im, s.re));
+                    s.im = fma(d.re, b.im, fma(d.im, b.re, s.im));
+                }
+                stc(&S.oslot[lsw(k)], s);
+            }
+        }
+        __syncthreads();                                  // bk[buf], rrows[buf] consumed; oslot complete
+        if (tid == 0) {
+            asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // dslot readable again (rows sent)
+            if (i + 2 < kn) {
+                mb_expect(&S.mbar_rows[buf], kL * 512 * 16);                  // rows of step i + 2
+                issue_bk_l(S, bkf, i + 2, o, buf);
+            }
+        }
+        if (warp < 2) {   // ---- C: inverse (warp pair 0), round, << 16 h ----
+            dcplx x[8];
+            inv2w(x, S.oslot, t1, t2, t3, tt, 4);
+#pragma unroll
+            for (int v = 0; v < 8; v++) {
+                const int c = gp1(tt, v);
+                S.res[c] = round_mod32(x[v].re) << (16 * h);
+                S.res[c + 512] = round_mod32(x[v].im) << (16 * h);
+            }
+        }
+        __syncthreads();
+        if (tid == 0) push_peer(res_dst + (uint32_t)(buf * kN * 4), S.res, kN * 4, res_mb + (uint32_t)(buf * 8));
+        mb_wait(&S.mbar_res[buf], par);
+        for (int c = tid; c < kN; c += kLThreads) {       // ACC[q] += lo + 2^16 hi (own half + the sibling's)
+            const uint32_t nv = S.acc[c] + S.res[c] + S.rres[buf][c];
+            S.acc[c] = nv;
+            S.acc[c + kN] = 0u - nv;
+            S.acc[c + 2 * kN] = nv;
+        }
+        __syncthreads();                                  // rres[buf] consumed
+        if (tid == 0) {
+            asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // res readable again
+            if (i + 2 < kn) mb_expect(&S.mbar_res[buf], kN * 4);            // the sibling's half of step i + 2
+        }
+        __syncthreads();
+    }
+    cl_sync();
+    if (gl < A.nlanes && h == 0) {   // a5: CTA (0, 0) holds ACC.a, CTA (1, 0) holds ACC.b
+        uint32_t* out = A.out + (int64_t)gl * A.out_stride;
+        if (q == 0) {
+            for (int j = tid; j < kN; j += kLThreads) out[j] = j == 0 ? S.acc[0] : 0u - S.acc[kN - j];
+        } else if (tid == 0) {
+            out[kN] = S.acc[0];
+        }
+    }
+}
+
+static int brl_attr() {
+    static bool attr = false;
+    if (!attr) {
+        if (cudaFuncSetAttribute(brl_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(BrlSmem)) !=
+            cudaSuccess)
+            return -1;
+        attr = true;
+    }
+    return 0;
+}
+
+// clusters of brl that are co-resident on the device (one wave of bootstraps; 32 measured on B200: the 4-SM
+// clusters must fit inside a GPC), or <= 0 on error
+int brl_wave_lanes() {
+    if (brl_attr()) return -1;
+    cudaLaunchConfig_t cfg = {};
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 4;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.gridDim = dim3(4 * 256);
+    cfg.blockDim = dim3(kLThreads);
+    cfg.dynamicSmemBytes = sizeof(BrlSmem);
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    int n = 0;
+    if (cudaOccupancyMaxActiveClusters(&n, brl_kernel, &cfg) != cudaSuccess) return -1;
+    return n;
+}
+
+int launch_brl(const BrArgs& A, const double2* bkf, const double2* twL, cudaStream_t st) {
+    const size_t smem = sizeof(BrlSmem);
+    static_assert(sizeof(BrlSmem) <= 232448, "brl shared memory");
+    if (brl_attr()) return -1;
+    if (A.nlanes <= 0) return 0;
+    brl_kernel<<<4 * A.nlanes, kLThreads, smem, st>>>(A, bkf, twL);
+    return 0;
+}
+
+}  // namespace tb

@@ -217,6 +217,10 @@ __device__ __forceinline__ void fft_inv(dcplx (&x)[16], double2* buf, const doub
     gs_stage_const<8, 1, 0>(x);       // stage 1
 }
 
+__device__ __forceinline__ double small_to_double(uint32_t v, double bias) {   // v < 2^31 exactly, minus bias
+    return __hiloint2double(0x43300000, (int)v) - (4503599627370496.0 + bias);
+}
+
 // exact integer value (|v| < 2^51) of a double that is within 0.5 of it, reduced mod 2^32
 __device__ __forceinline__ uint32_t round_mod32(double v) {
     return (uint32_t)__double2loint(v + 6755399441055744.0);   // 1.5 * 2^52: mantissa holds v + 2^51

@@ -62,12 +62,16 @@ struct tb_ctx {
     int variant = 6;                        // blind-rotation kernel: 6 = br6, 7 = br7 (TMA-staged BK), 8 = br8
     int ks_tile = 8;                        // gates per key-switch CTA (8, 16, 32); 8 measured fastest
     int narrow_lanes = 0;                   // launches with <= this many lanes run in latency mode (= SM count)
-    int narrow_kernel = 9;                  // latency-mode kernel: 9 = br9 (2-SM cluster per lane), 7 = br7<1>
+    int narrow_kernel = 0;                  // latency-mode kernel: 9 = br9 (2-SM cluster per lane), 7 = br7<1>,
+                                            // 11 = brl (4-SM cluster per lane, FP64 path), 0 = auto:
+                                            // brl while the lanes fit in one wave of its clusters, else br9
+    int brl_wave = -2;                      // co-resident brl clusters (queried on first use)
     cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
     uint2* twF = nullptr;                   // [31][32]
     uint2* twI = nullptr;
     double2* fftB = nullptr;                // FP64 FFT per-lane twiddles: stages 5-8 [15][32], stage 9 [8][32]
     double2* fftC = nullptr;
+    double2* fftL = nullptr;                // brl: [64][6] per-thread pass-2/3 twiddle bases
     uint32_t ninv = 0, ninvp = 0;
     uint32_t* bkhat = nullptr;              // [n][6][6][N]
     double2* bkf = nullptr;                 // FP64 variant: [n][6][4][512] complex, scaled by 1/512
@@ -217,6 +221,16 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
     for (int s = 5; s <= 8; s++)
         for (int u = 0; u < 16; u++) fb[(s - 5) * 16 + u] = cpsi(brv10((1u << s) + (uint32_t)u * (1u << (s - 5))));
     for (int t = 0; t < 32; t++) fc[t] = cpsi(brv10(512u + (uint32_t)t * 8u));
+    std::vector<double2> fl(64 * 6);       // brl pass bases (tb_brl.cu): zeta_{s,b} = psi^brv10(2^s + b)
+    for (int t = 0; t < 64; t++) {
+        const uint32_t T = (uint32_t)t >> 3;
+        fl[t * 6 + 0] = cpsi(brv10(16u + T));
+        fl[t * 6 + 1] = cpsi(brv10(32u + 2 * T));
+        fl[t * 6 + 2] = cpsi(brv10(64u + 4 * T));
+        fl[t * 6 + 3] = cpsi(brv10(128u + (uint32_t)t));
+        fl[t * 6 + 4] = cpsi(brv10(256u + 2 * (uint32_t)t));
+        fl[t * 6 + 5] = cpsi(brv10(512u + 4 * (uint32_t)t));
+    }
     c->ninv = powmod(kN, kP - 2);
     c->ninvp = shoup_of(c->ninv);
     int rc = set_ntt_constants(fw, fwp, iw, iwp, misc);
@@ -226,6 +240,8 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
     if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->fftC, fc.size() * sizeof(double2));
     if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->fftB, fb.data(), fb.size() * sizeof(double2), cudaMemcpyHostToDevice);
     if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->fftC, fc.data(), fc.size() * sizeof(double2), cudaMemcpyHostToDevice);
+    if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->fftL, fl.size() * sizeof(double2));
+    if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->fftL, fl.data(), fl.size() * sizeof(double2), cudaMemcpyHostToDevice);
     if (rc == 0 && e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->own, cudaStreamNonBlocking);
     if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->twF, 31 * 32 * sizeof(uint2));
     if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->twI, 31 * 32 * sizeof(uint2));
@@ -246,6 +262,7 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
     cudaFree(c->twI);
     cudaFree(c->fftB);
     cudaFree(c->fftC);
+    cudaFree(c->fftL);
     cudaFree(c->bkhat);
     cudaFree(c->bkf);
     cudaFree(c->ksk);
@@ -276,7 +293,8 @@ extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
 }
 
 extern "C" int tb_set_narrow_kernel(tb_ctx* c, int kernel) {
-    if (!c || (kernel != 7 && kernel != 9)) return fail(TB_EINVAL, "latency-mode kernel must be 7 or 9");
+    if (!c || (kernel != 0 && kernel != 7 && kernel != 9 && kernel != 11))
+        return fail(TB_EINVAL, "latency-mode kernel must be 0 (auto), 7, 9 or 11");
     c->narrow_kernel = kernel;
     return TB_OK;
 }
@@ -380,9 +398,15 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     A.out = out; A.out_stride = ostride;
     const long slot = prof_begin(c, 0, st);
     int rc;
+    int nk = c->narrow_kernel;
+    if (nk == 0) {   // auto: measured one-lane level 2.2 ms (brl) vs 4.2 ms (br9), 32 vs 74 lanes per wave
+        if (c->brl_wave == -2) c->brl_wave = brl_wave_lanes();
+        nk = nlanes <= c->brl_wave ? 11 : 9;
+    }
     if (c->narrow_lanes > 0 && nlanes <= c->narrow_lanes)
-        rc = c->narrow_kernel == 9 ? launch_br9(A, st)   // narrow level: one lane per 2-SM cluster
-                                   : launch_br7(A, 1, st);  // or one lane per SM, BK staged per step
+        rc = nk == 9    ? launch_br9(A, st)                    // narrow level: one lane per 2-SM cluster
+             : nk == 11 ? launch_brl(A, c->bkf, c->fftL, st)   // or per 4-SM cluster (FP64)
+                                      : launch_br7(A, 1, st);                // or one lane per SM
     else if (c->variant == 7)
         rc = launch_br7(A, 2, st);
     else if (c->variant == 10)

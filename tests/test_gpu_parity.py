@@ -89,20 +89,21 @@ def test_bootstrap_wo_ks_bit_exact(tb, ctx, keys):
         assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), k
 
 
-@pytest.mark.parametrize("kernel", [9, 7])
+@pytest.mark.parametrize("kernel", [0, 9, 7, 11])
 def test_narrow_level_latency_mode_bit_exact(tb, ctx, keys, kernel):
-    """small launches run the latency kernel (br9: 2-SM cluster per lane, or br7<1>: one SM per lane);
-    149 lanes fall back to the throughput kernel"""
+    """small launches run the latency kernel (br9: 2-SM cluster per lane, br7<1>: one SM per lane, brl: 4-SM
+    cluster per lane on the FP64 path; 40 lanes = 160 CTAs is more than one wave); 149 lanes fall back to the
+    throughput kernel"""
     rng = np.random.default_rng(39 + kernel)
     ctx.set_narrow_kernel(kernel)
     try:
-        for count in (1, 3, 149):
+        for count in (1, 3, 40, 149):
             cts = rng.integers(0, M32, (count, 631), dtype=np.uint64).astype(np.uint32)
             got = ctx.bootstrap_wo_ks(ctx.to_device(cts))[:, :1025].cpu().numpy().view(np.uint32)
             for k in sorted({0, count - 1}):
                 assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), (count, k)
     finally:
-        ctx.set_narrow_kernel(9)
+        ctx.set_narrow_kernel(0)
 
 
 @pytest.mark.parametrize("variant", [6, 7, 8, 10])
