@@ -58,7 +58,7 @@ __device__ __forceinline__ void mbar_expect9(unsigned long long* bar, uint32_t b
 }
 __device__ __forceinline__ void mbar_wait9(unsigned long long* bar, uint32_t parity) {
     asm volatile(
-        "{\n .reg .pred p;\n W9_%=:\n mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n"
+        "{\n .reg .pred p;\n W9_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
         " @!p bra W9_%=;\n}\n" ::"r"(smem_u32_9(bar)),
         "r"(parity)
         : "memory");

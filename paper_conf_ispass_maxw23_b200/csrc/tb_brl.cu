@@ -145,7 +145,7 @@ __device__ __forceinline__ void mb_expect(unsigned long long* b, uint32_t bytes)
 }
 __device__ __forceinline__ void mb_wait(unsigned long long* b, uint32_t parity) {
     asm volatile(
-        "{\n .reg .pred p;\n WL_%=:\n mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n"
+        "{\n .reg .pred p;\n WL_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
         " @!p bra WL_%=;\n}\n" ::"r"(sm32(b)),
         "r"(parity)
         : "memory");
