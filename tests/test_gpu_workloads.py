@@ -163,3 +163,39 @@ def test_errors_without_keys_and_bad_arguments(tb):
     with pytest.raises(ValueError):
         c.gates(tb.NAND, x, x[:, :600])                           # shape mismatch caught in the binding
     c.close()
+
+
+@pytest.mark.parametrize("fmt", ["yosys", "blif"])
+def test_imported_netlist_bit_exact(tb, ctx, keys, fmt):
+    """a synthesised gate-level netlist (Yosys JSON / BLIF fixture) imported, run on the GPU for
+    all 8 input assignments at once (8 copies side by side), every wire equal to the oracle's, outputs decrypt to
+    the full adder"""
+    import itertools
+    import os
+    from oracle.algorithm1 import algorithm1
+    from paper_conf_ispass_maxw23_b200 import netlist as NL
+    gold = os.path.join(os.path.dirname(__file__), "golden")
+    net = (NL.read_yosys_json(open(os.path.join(gold, "full_adder_yosys.json")).read()) if fmt == "yosys"
+           else NL.read_blif(open(os.path.join(gold, "full_adder.blif")).read()))
+    # 8 disjoint copies of the netlist in one program (copy k uses inputs 3k .. 3k+2)
+    k8, ni, ng = 8, net.n_inputs, net.n_gates
+    remap = lambda w, k: np.where(w < 0, -1, np.where(w < ni, w + k * ni, k8 * ni + k * ng + (w - ni)))
+    n = dict(n_inputs=k8 * ni, type=np.tile(net.type, k8),
+             in0=np.concatenate([remap(net.in0, k) for k in range(k8)]),
+             in1=np.concatenate([remap(net.in1, k) for k in range(k8)]),
+             in2=np.concatenate([remap(net.in2, k) for k in range(k8)]),
+             outputs=np.concatenate([remap(net.outputs, k) for k in range(k8)]))
+    bits = np.array(list(itertools.product((0, 1), repeat=3)), np.uint8).reshape(-1)
+    cts = O.encrypt_bits(keys, bits, 31)
+    w, _ = run(tb, ctx, n, cts)
+    ref = np.zeros_like(w)
+    ref[:n["n_inputs"]] = cts
+    for batch in algorithm1(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"]):
+        b = np.array(batch)
+        O.run_level(keys, ref, n["type"][b], n["in0"][b], n["in1"][b], n["in2"][b], n["n_inputs"] + b)
+    assert (w == ref).all()
+    dec = O.decrypt_bits(keys, w[n["outputs"]]).reshape(k8, -1)
+    plain = simulate(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"], bits)[0][n["outputs"]].reshape(k8, -1)
+    assert (dec == plain).all()
+    a, b_, c = bits.reshape(k8, 3).T.astype(int)
+    assert (dec[:, 0] == (a ^ b_ ^ c)).all() and (dec[:, 1] == ((a & b_) | (c & (a ^ b_)))).all()
