@@ -108,6 +108,10 @@ int tb_levelise(const tb_netlist* net, int64_t* level_of_gate, int64_t* n_levels
  * level).  Pass level_off = row_of_wire = NULL to query n_levels first.  This is the layout
  * tb_netlist_upload uses and the one the multi-GPU level loop shards (contiguous output rows per level). */
 int tb_netlist_plan(const tb_netlist* net, int64_t* n_levels, int64_t* level_off, int64_t* row_of_wire);
+/* tb_netlist_plan with the capacity-aware level schedule of tb_set_level_capacity (`lanes` > 0; 0 = Algorithm 1,
+ * i.e. tb_netlist_plan).  Host only.  lanes < 0: TB_EINVAL. */
+int tb_netlist_plan_capacity(const tb_netlist* net, int64_t lanes, int64_t* n_levels, int64_t* level_off,
+                             int64_t* row_of_wire);
 
 typedef struct tb_dev_netlist tb_dev_netlist;   /* library-owned device copy of a levelised netlist */
 
@@ -178,6 +182,13 @@ int tb_set_narrow_lanes(tb_ctx* ctx, int64_t lanes);
  * rows exchanged through distributed shared memory; 4.2 ms), 7 = br7<1> (one bootstrap per SM).  All are
  * bit-identical.  Anything else: TB_EINVAL. */
 int tb_set_narrow_kernel(tb_ctx* ctx, int kernel);
+/* Level schedule used by tb_netlist_upload: Algorithm 1 gives every gate its earliest level;
+ * with lanes > 0 gates that have slack are moved to later levels (never past their latest level, so the number
+ * of levels is unchanged) to keep each level within `lanes` bootstraps (MUX = 2, NOT = 0) where possible: a
+ * narrow level then fits one wave of the latency kernel.  -1 = auto (default; the number of brl clusters that
+ * fit on the device, 32 on B200), 0 = Algorithm 1 as is.  Output bytes are identical either way (each gate's
+ * result depends only on its inputs).  Affects netlists uploaded afterwards.  lanes < -1: TB_EINVAL. */
+int tb_set_level_capacity(tb_ctx* ctx, int64_t lanes);
 /* Gates per key-switch CTA (8, 16 or 32; default 8): each tile streams the 62 MB KSK once from L2. */
 int tb_set_ks_tile(tb_ctx* ctx, int gates);
 /* Device bytes a context holds for keys (BK NTT + KSK). */

@@ -123,11 +123,15 @@ class Context:
         _native.check(_native.lib().tb_set_br_variant(self._h, variant))
 
     def set_narrow_lanes(self, lanes: int):
-        """levels with <= lanes bootstraps run in latency mode (br7, one lane per SM); 0 disables"""
+        """levels with <= lanes bootstraps run in latency mode (see set_narrow_kernel); 0 disables"""
         _native.check(_native.lib().tb_set_narrow_lanes(self._h, lanes))
 
+    def set_level_capacity(self, lanes: int):
+        """netlist uploads: keep levels within `lanes` bootstraps where slack allows (-1 auto, 0 = Algorithm 1)"""
+        _native.check(_native.lib().tb_set_level_capacity(self._h, lanes))
+
     def set_narrow_kernel(self, kernel: int):
-        """latency-mode kernel: 9 = br9 (2-SM cluster per bootstrap, default), 7 = br7<1> (one SM)"""
+        """latency-mode kernel: 0 = auto (default), 11 = brl (4-SM cluster), 9 = br9 (2-SM cluster), 7 = br7<1>"""
         _native.check(_native.lib().tb_set_narrow_kernel(self._h, kernel))
 
     def set_ks_tile(self, gates: int):

@@ -72,6 +72,7 @@ SIGNATURES = {
     "tb_gates_host": (ctypes.c_int, [_vp, ctypes.c_int, _vp, _vp, _vp, _vp, _i64, _i64]),
     "tb_levelise": (ctypes.c_int, [ctypes.POINTER(Netlist), _vp, _pi64]),
     "tb_netlist_plan": (ctypes.c_int, [ctypes.POINTER(Netlist), _pi64, _vp, _vp]),
+    "tb_netlist_plan_capacity": (ctypes.c_int, [ctypes.POINTER(Netlist), _i64, _pi64, _vp, _vp]),
     "tb_netlist_upload":(ctypes.c_int, [_vp, ctypes.POINTER(Netlist), ctypes.POINTER(_vp)]),
     "tb_netlist_free": (ctypes.c_int, [_vp, _vp]),
     "tb_netlist_info": (ctypes.c_int, [_vp, _pi64, _pi64]),
@@ -92,6 +93,7 @@ SIGNATURES = {
     "tb_set_ks_tile": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_set_narrow_lanes": (ctypes.c_int, [_vp, _i64]),
     "tb_set_narrow_kernel": (ctypes.c_int, [_vp, ctypes.c_int]),
+    "tb_set_level_capacity": (ctypes.c_int, [_vp, _i64]),
     "tb_key_bytes": (ctypes.c_int, [_vp, ctypes.POINTER(_sz)]),
     "tb_microbench": (ctypes.c_int, [_vp, ctypes.c_int, ctypes.POINTER(ctypes.c_double),
                                      ctypes.POINTER(ctypes.c_double)]),

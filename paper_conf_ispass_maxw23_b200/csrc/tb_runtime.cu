@@ -66,6 +66,8 @@ struct tb_ctx {
                                             // 11 = brl (4-SM cluster per lane, FP64 path), 0 = auto:
                                             // brl while the lanes fit in one wave of its clusters, else br9
     int brl_wave = -2;                      // co-resident brl clusters (queried on first use)
+    int64_t level_capacity = -1;            // netlist upload: re-levelise to <= this many lanes per level where
+                                            // slack allows (0 = Algorithm 1 as is, -1 = auto: brl_wave)
     cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
     uint2* twF = nullptr;                   // [31][32]
     uint2* twI = nullptr;
@@ -296,6 +298,12 @@ extern "C" int tb_set_narrow_kernel(tb_ctx* c, int kernel) {
     if (!c || (kernel != 0 && kernel != 7 && kernel != 9 && kernel != 11))
         return fail(TB_EINVAL, "latency-mode kernel must be 0 (auto), 7, 9 or 11");
     c->narrow_kernel = kernel;
+    return TB_OK;
+}
+
+extern "C" int tb_set_level_capacity(tb_ctx* c, int64_t lanes) {
+    if (!c || lanes < -1) return fail(TB_EINVAL, "level capacity must be -1 (auto), 0 (off) or > 0");
+    c->level_capacity = lanes;
     return TB_OK;
 }
 
@@ -634,15 +642,76 @@ extern "C" int tb_levelise(const tb_netlist* net, int64_t* level_of_gate, int64_
     return TB_OK;
 }
 
-// Levelise (Algorithm 1) and renumber: inputs keep rows [0, n_inputs); the gates of level L follow those of
-// level L-1, ascending original index inside a level.  level_off (0-based, n_levels + 1 entries) are gate
-// offsets into that order; order[k] = original gate index of the k-th gate.
+// Capacity-aware re-levelisation ("dependency-driven scheduling beyond strict levels").
+// Algorithm 1 runs every gate at its earliest level (ASAP).  On a deep, narrow netlist a level whose
+// bootstraps exceed one wave of the latency kernel costs a second wave although many of its gates have
+// slack.  Here each gate g has a window [ASAP(g), ALAP(g)] (ALAP = latest level that keeps the depth); levels
+// are built in order: every ready gate whose deadline is this level is taken, then ready gates by increasing
+// deadline while the level's lanes (MUX = 2 bootstraps, NOT = 0) stay <= `cap`.  The depth is unchanged
+// (every gate runs by its deadline), so the serial chain of levels is as short as Algorithm 1's.
+static void relevel_capacity(const tb_netlist* net, std::vector<int64_t>& lv, int64_t nlev, int64_t cap) {
+    const int64_t ni = net->n_inputs, ng = net->n_gates;
+    auto need = [&](int64_t g, int k) {
+        const int t = net->type[g];
+        return k == 0 || (k == 1 && t != TB_NOT) || (k == 2 && t == TB_MUX);
+    };
+    auto src = [&](int64_t g, int k) { return k == 0 ? net->in0[g] : (k == 1 ? net->in1[g] : net->in2[g]); };
+    // successor lists (gate -> consumers) and ALAP by a reverse sweep over the ASAP order
+    std::vector<int64_t> head((size_t)ng + 1, 0), adj, pend((size_t)ng, 0);
+    for (int64_t g = 0; g < ng; g++)
+        for (int k = 0; k < 3; k++)
+            if (need(g, k) && src(g, k) >= ni) { head[src(g, k) - ni + 1]++; pend[g]++; }
+    for (int64_t g = 0; g < ng; g++) head[g + 1] += head[g];
+    adj.resize((size_t)head[ng]);
+    std::vector<int64_t> fill(head.begin(), head.end() - 1);
+    for (int64_t g = 0; g < ng; g++)
+        for (int k = 0; k < 3; k++)
+            if (need(g, k) && src(g, k) >= ni) adj[fill[src(g, k) - ni]++] = g;
+    std::vector<int64_t> byl((size_t)ng);
+    for (int64_t g = 0; g < ng; g++) byl[g] = g;
+    std::stable_sort(byl.begin(), byl.end(), [&](int64_t x, int64_t y) { return lv[x] > lv[y]; });
+    std::vector<int64_t> alap((size_t)ng, nlev);
+    for (int64_t g : byl)
+        for (int64_t e = head[g]; e < head[g + 1]; e++) alap[g] = std::min(alap[g], alap[adj[e]] - 1);
+    auto lanes = [&](int64_t g) { return net->type[g] == TB_MUX ? 2 : (net->type[g] == TB_NOT ? 0 : 1); };
+    std::vector<std::vector<int64_t>> bucket((size_t)nlev + 2);    // ready gates by deadline
+    for (int64_t g = 0; g < ng; g++)
+        if (pend[g] == 0) bucket[alap[g]].push_back(g);
+    std::vector<int64_t> took;
+    for (int64_t L = 1; L <= nlev; L++) {
+        took.clear();
+        int64_t used = 0;
+        for (int64_t g : bucket[L]) { took.push_back(g); used += lanes(g); }   // deadline now: always
+        bucket[L].clear();
+        for (int64_t a = L + 1; a <= nlev && used < cap; a++) {
+            auto& B = bucket[a];
+            size_t keep = 0;
+            for (size_t j = 0; j < B.size(); j++) {
+                const int64_t g = B[j];
+                if (used + lanes(g) <= cap) { took.push_back(g); used += lanes(g); }
+                else B[keep++] = g;
+            }
+            B.resize(keep);
+        }
+        for (int64_t g : took) {
+            lv[g] = L;
+            for (int64_t e = head[g]; e < head[g + 1]; e++)
+                if (--pend[adj[e]] == 0) bucket[alap[adj[e]]].push_back(adj[e]);
+        }
+    }
+}
+
+// Levelise (Algorithm 1, then capacity-aware re-levelisation when cap > 0) and renumber: inputs keep rows
+// [0, n_inputs); the gates of level L follow those of level L-1, ascending original index inside a level.
+// level_off (0-based, n_levels + 1 entries) are gate offsets into that order; order[k] = original gate index
+// of the k-th gate.
 static int plan_impl(const tb_netlist* net, int64_t* n_levels, std::vector<int64_t>& level_off,
-                     std::vector<int64_t>& order, std::vector<int64_t>& row_of_wire) {
+                     std::vector<int64_t>& order, std::vector<int64_t>& row_of_wire, int64_t cap = 0) {
     std::vector<int64_t> lv;
     int64_t nlev = 0;
     int rc = levelise_impl(net, lv, &nlev);
     if (rc) return rc;
+    if (cap > 0) relevel_capacity(net, lv, nlev, cap);
     const int64_t ni = net->n_inputs, ng = net->n_gates;
     std::vector<int64_t> cnt((size_t)nlev + 2, 0);
     for (int64_t g = 0; g < ng; g++) cnt[lv[g]]++;
@@ -659,9 +728,15 @@ static int plan_impl(const tb_netlist* net, int64_t* n_levels, std::vector<int64
 }
 
 extern "C" int tb_netlist_plan(const tb_netlist* net, int64_t* n_levels, int64_t* level_off, int64_t* row_of_wire) {
+    return tb_netlist_plan_capacity(net, 0, n_levels, level_off, row_of_wire);
+}
+
+extern "C" int tb_netlist_plan_capacity(const tb_netlist* net, int64_t lanes, int64_t* n_levels, int64_t* level_off,
+                                        int64_t* row_of_wire) {
     if (!net || !n_levels) return fail(TB_EINVAL, "null argument");
+    if (lanes < 0) return fail(TB_EINVAL, "capacity must be >= 0");
     std::vector<int64_t> lo, order, rows;
-    int rc = plan_impl(net, n_levels, lo, order, rows);
+    int rc = plan_impl(net, n_levels, lo, order, rows, lanes);
     if (rc) return rc;
     if (level_off) std::copy(lo.begin(), lo.end(), level_off);
     if (row_of_wire) std::copy(rows.begin(), rows.end(), row_of_wire);
@@ -675,7 +750,12 @@ extern "C" int tb_netlist_upload(tb_ctx* c, const tb_netlist* net, tb_dev_netlis
     tb_dev_netlist* d = new (std::nothrow) tb_dev_netlist();
     if (!d) return fail(TB_ENOMEM, "host allocation failed");
     std::vector<int64_t> order;
-    int rc = plan_impl(net, &d->n_levels, d->level_off, order, d->row_of_wire);
+    int64_t cap = c->level_capacity;
+    if (cap < 0) {   // auto: one wave of the latency kernel brl (32 bootstraps on B200)
+        if (c->brl_wave == -2) c->brl_wave = brl_wave_lanes();
+        cap = c->brl_wave > 0 ? c->brl_wave : 0;
+    }
+    int rc = plan_impl(net, &d->n_levels, d->level_off, order, d->row_of_wire, cap);
     if (rc) {
         delete d;
         return rc;

@@ -63,16 +63,17 @@ class Netlist:
         _native.check(_native.lib().tb_levelise(ctypes.byref(s), lv.ctypes.data, ctypes.byref(nl)))
         return lv, int(nl.value)
 
-    def plan(self):
-        """Host-only execution plan (tb_netlist_plan): (levels [(row0, n_gates)], row_of_wire int64).  Level L's
-        outputs are rows row0 .. row0 + n_gates - 1 of the wire array (contiguous, as the all-gather needs)."""
+    def plan(self, capacity: int = 0):
+        """Host-only execution plan (tb_netlist_plan_capacity): (levels [(row0, n_gates)], row_of_wire int64).
+        Level L's outputs are rows row0 .. row0 + n_gates - 1 of the wire array (contiguous, as the all-gather
+        needs).  capacity > 0: the capacity-aware level schedule (f1) that tb_netlist_upload uses."""
         s = self.c_struct()
         nl = ctypes.c_int64(0)
-        _native.check(_native.lib().tb_netlist_plan(ctypes.byref(s), ctypes.byref(nl), None, None))
+        f = _native.lib().tb_netlist_plan_capacity
+        _native.check(f(ctypes.byref(s), capacity, ctypes.byref(nl), None, None))
         off = np.zeros(int(nl.value) + 1, np.int64)
         rows = np.zeros(self.n_wires, np.int64)
-        _native.check(_native.lib().tb_netlist_plan(ctypes.byref(s), ctypes.byref(nl), off.ctypes.data,
-                                                    rows.ctypes.data))
+        _native.check(f(ctypes.byref(s), capacity, ctypes.byref(nl), off.ctypes.data, rows.ctypes.data))
         levels = [(self.n_inputs + int(off[L]), int(off[L + 1] - off[L])) for L in range(int(nl.value))]
         return levels, rows
 

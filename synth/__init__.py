@@ -9,6 +9,7 @@ and (c) gate netlists with the shapes of the paper's workloads (DESIGN.md "Input
   cfg 3  one level of G independent NAND/XOR gates (configs[2], the throughput sweep)
   cfg 4  VIP-Bench-shaped 32x32 multiplier / bubble sort of 16 x 16-bit (configs[3])
   cfg 5  ChiselTorch-shaped 8-bit MNIST MLP tile (configs[4])
+  f3     self-attention layer shaped like Attention_S / Attention_L
 Netlists are returned as plain arrays: (n_inputs, type int32, in0/in1/in2 int64, outputs int64); wire ids
 [0, n_inputs) are inputs and n_inputs + g is gate g's output.  Gate codes follow reading C15.
 """
@@ -258,6 +259,84 @@ def mnist_fig4(side: int = 26, bits: int = 8, n_out: int = 10, pool: int = 3):
             prods = nxt
         outs += prods[0]
     return B.arrays(outs)
+
+
+def _mul(B: Builder, x, y):
+    """unsigned array multiply of LSB-first lists (AND partial products, ripple rows)"""
+    rows = [[B.gate(AND, x[k], y[j]) for k in range(len(x))] for j in range(len(y))]
+    acc = rows[0]
+    for j in range(1, len(y)):
+        acc = acc[:j] + _add(B, acc[j:], rows[j])
+    return acc
+
+
+def _dot(B: Builder, xs, ys):
+    """sum_i xs[i] * ys[i] (array multipliers + adder tree)"""
+    prods = [_mul(B, x, y) for x, y in zip(xs, ys)]
+    while len(prods) > 1:
+        nxt = [_add(B, prods[k], prods[k + 1]) for k in range(0, len(prods) - 1, 2)]
+        if len(prods) % 2:
+            nxt.append(prods[-1])
+        prods = nxt
+    return prods[0]
+
+
+def attention(seq: int = 4, hidden: int = 32, bits: int = 4):
+    """f3: a self-attention layer shaped like the paper's Attention_S / Attention_L (hidden 32 /
+    64), built from Table I primitives (matmul, argmax, +, *) on encrypted `bits`-bit unsigned
+    tokens X [seq][hidden] and encrypted weights Wq, Wk, Wv [hidden][hidden]:
+        Q, K, V = requant(X Wq), requant(X Wk), requant(X Wv)      requant(z) = top `bits` bits of the
+                                                                   (2 bits + ceil(log2 hidden))-bit dot product
+        S = Q K^T;  out[i] = V[argmax_j S[i][j]]                   (hard attention: argmax in place of softmax,
+                                                                   the first maximum wins)
+    The paper gives neither the sequence length nor the number format, so both are parameters.  Inputs: X, then
+    Wq, Wk, Wv (row-major, LSB first); outputs out [seq][hidden] (LSB first).  attention_reference() is the same
+    function on plaintext integers."""
+    w_full = 2 * bits + max(1, (hidden - 1).bit_length())
+    n_in = seq * hidden * bits + 3 * hidden * hidden * bits
+    B = Builder(n_in)
+    word = lambda base, i: list(range(base + i * bits, base + (i + 1) * bits))
+    X = [[word(0, t * hidden + h) for h in range(hidden)] for t in range(seq)]
+    W = []
+    for m in range(3):
+        base = seq * hidden * bits + m * hidden * hidden * bits
+        W.append([[word(base, r * hidden + c) for c in range(hidden)] for r in range(hidden)])
+
+    def requant(z):
+        if len(z) != w_full:
+            raise ValueError("dot-product width %d, expected %d (hidden must be a power of two)" % (len(z), w_full))
+        return z[w_full - bits:]
+
+    proj = [[[requant(_dot(B, X[t], [W[m][r][c] for r in range(hidden)])) for c in range(hidden)]
+             for t in range(seq)] for m in range(3)]
+    Q, K, V = proj
+    outs = []
+    for i in range(seq):
+        cands = [(_dot(B, Q[i], K[j]), V[j]) for j in range(seq)]
+        while len(cands) > 1:                          # argmax tournament, earlier index wins ties
+            nxt = []
+            for k in range(0, len(cands) - 1, 2):
+                (s1, v1), (s2, v2) = cands[k], cands[k + 1]
+                take2 = _less_than(B, s1, s2)                   # all scores have the same width
+                s = [B.gate(MUX, take2, s2[b], s1[b]) for b in range(len(s1))]
+                v = [[B.gate(MUX, take2, v2[h][b], v1[h][b]) for b in range(bits)] for h in range(hidden)]
+                nxt.append((s, v))
+            if len(cands) % 2:
+                nxt.append(cands[-1])
+            cands = nxt
+        outs += [b for h in cands[0][1] for b in h]
+    return B.arrays(outs)
+
+
+def attention_reference(x, wq, wk, wv, bits: int):
+    """plaintext integers of attention(): x [seq][hidden], w* [hidden][hidden] -> out [seq][hidden]"""
+    x, wq, wk, wv = (np.asarray(a, np.int64) for a in (x, wq, wk, wv))
+    hidden = x.shape[1]
+    w_full = 2 * bits + max(1, (hidden - 1).bit_length())
+    rq = lambda z: (z >> (w_full - bits)) & ((1 << bits) - 1)
+    q, k, v = rq(x @ wq), rq(x @ wk), rq(x @ wv)
+    s = q @ k.T
+    return v[np.argmax(s, axis=1)]
 
 
 def pack_bits(values, bits: int) -> np.ndarray:

@@ -199,3 +199,18 @@ def test_imported_netlist_bit_exact(tb, ctx, keys, fmt):
     assert (dec == plain).all()
     a, b_, c = bits.reshape(k8, 3).T.astype(int)
     assert (dec[:, 0] == (a ^ b_ ^ c)).all() and (dec[:, 1] == ((a & b_) | (c & (a ^ b_)))).all()
+
+
+def test_attention_f3(tb, ctx, keys):
+    """a small Attention layer (seq 2, hidden 4, 3-bit; 5,866 gates incl. 40 MUX) on the GPU:
+    outputs decrypt to the plaintext hard self-attention, 64 seeded gates bit-exact vs the oracle"""
+    seq, hidden, bits = 2, 4, 3
+    n = synth.attention(seq, hidden, bits)
+    rng = np.random.default_rng(12)
+    x, wq, wk, wv = rng.integers(0, 8, (seq, hidden)), *(rng.integers(0, 8, (hidden, hidden)) for _ in range(3))
+    pbits = np.concatenate([synth.pack_bits(a.reshape(-1), bits) for a in (x, wq, wk, wv)])
+    cts = O.encrypt_bits(keys, pbits, 13)
+    w, _ = run(tb, ctx, n, cts)
+    dec = O.decrypt_bits(keys, w[n["outputs"]])
+    assert (synth.unpack_bits(dec, bits).reshape(seq, hidden) == synth.attention_reference(x, wq, wk, wv, bits)).all()
+    sampled_gate_parity(keys, n, w, 64, 14)

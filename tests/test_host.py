@@ -225,7 +225,103 @@ def test_mnist_fig4_full_size_shape(tb):
     assert w[w >= 8192].sum() / w.sum() > 0.9
 
 
+@pytest.mark.parametrize("seq,hidden,bits", [(3, 4, 3), (2, 8, 2), (4, 2, 3)])
+def test_attention_computes_hard_self_attention(seq, hidden, bits):
+    """the gate-level Attention layer equals its plaintext integer definition (requantised
+    projections, Q K^T, first-maximum argmax, V row select), on random tokens/weights and on tie cases"""
+    n = synth.attention(seq, hidden, bits)
+    rng = np.random.default_rng(seq * 100 + hidden)
+    cases = [tuple(rng.integers(0, 1 << bits, sh) for sh in [(seq, hidden)] + [(hidden, hidden)] * 3) for _ in range(5)]
+    z = np.zeros((hidden, hidden), np.int64)
+    cases.append((rng.integers(0, 1 << bits, (seq, hidden)), z, z, rng.integers(0, 1 << bits, (hidden, hidden))))
+    for x, wq, wk, wv in cases:                       # the last case: all scores 0, so argmax = 0 everywhere
+        bitsv = np.concatenate([synth.pack_bits(a.reshape(-1), bits) for a in (x, wq, wk, wv)])
+        got = synth.unpack_bits(_eval(n, bitsv[None])[0], bits).reshape(seq, hidden)
+        assert (got == synth.attention_reference(x, wq, wk, wv, bits)).all()
+
+
+def test_attention_paper_sizes(tb):
+    """Attention_S / Attention_L shapes (hidden 32 / 64) at seq 4, 4-bit: ~1.3 M / ~5.3 M gates"""
+    for hidden, lo, hi in ((32, 1_000_000, 2_000_000), (64, 4_000_000, 7_000_000)):
+        n = synth.attention(4, hidden, 4)
+        assert lo < len(n["type"]) < hi
+        assert len(n["outputs"]) == 4 * hidden * 4
+
+
 def test_independent_level_shape():
     n = synth.independent_level(64, 5)
     assert n["n_inputs"] == 128 and set(np.unique(n["type"]).tolist()) <= {6, 7}
     assert len(set(n["in0"].tolist()) | set(n["in1"].tolist())) == 128
+
+
+# ------------------------------------------------------------------- f1: capacity-aware level schedule
+def _sched(net, cap):
+    levels, rows = net.plan(cap)
+    lv = np.zeros(net.n_gates, np.int64)
+    for L, (row0, cnt) in enumerate(levels, 1):
+        g = np.where((rows[net.n_inputs:] >= row0) & (rows[net.n_inputs:] < row0 + cnt))[0]
+        lv[g] = L
+    return levels, rows, lv
+
+
+@pytest.mark.parametrize("shape", ["mul", "sort", "rca", "random"])
+def test_capacity_schedule_is_valid_and_keeps_depth(tb, shape):
+    """same number of levels as Algorithm 1, every gate after all its inputs, and a level that
+    exceeds the capacity holds only gates at their deadline (latest level that keeps the depth)"""
+    if shape == "random":
+        r = np.random.default_rng(9)
+        n_in, ng = 20, 600
+        t = r.choice([1, 3, 6, 7, 8, 16], ng).astype(np.int32)
+        a = np.array([r.integers(0, n_in + g) for g in range(ng)])
+        b = np.array([r.integers(0, n_in + g) for g in range(ng)])
+        c = np.where(t == 16, [r.integers(0, n_in + g) for g in range(ng)], -1)
+        n = dict(n_inputs=n_in, type=t, in0=a, in1=np.where(t == 3, -1, b), in2=c, outputs=np.arange(ng) + n_in)
+    else:
+        n = {"mul": lambda: synth.array_multiplier(12), "sort": lambda: synth.bubble_sort(8, 6),
+             "rca": lambda: synth.ripple_carry_adder(8)}[shape]()
+    net = tb.Netlist(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"], outputs=n["outputs"])
+    asap, depth = net.levels()
+    cap = 8
+    levels, rows, lv = _sched(net, cap)
+    assert len(levels) == depth
+    ni = net.n_inputs
+    lvl_of = lambda w: 0 if w < ni else lv[w - ni]
+    for g in range(net.n_gates):
+        ins = [net.in0[g]] + ([net.in1[g]] if net.type[g] != 3 else []) + ([net.in2[g]] if net.type[g] == 16 else [])
+        assert all(lvl_of(w) < lv[g] for w in ins), g
+    assert (lv >= asap).all()
+    # deadlines: ALAP by a reverse sweep
+    alap = np.full(net.n_gates, depth)
+    for g in np.argsort(-asap, kind="stable"):
+        for w in [net.in0[g], net.in1[g], net.in2[g]]:
+            if w >= ni and (w != net.in1[g] or net.type[g] != 3) and (w != net.in2[g] or net.type[g] == 16):
+                alap[w - ni] = min(alap[w - ni], alap[g] - 1)
+    assert (lv <= alap).all()
+    lanes = np.where(net.type == 16, 2, np.where(net.type == 3, 0, 1))
+    for L in range(1, depth + 1):
+        m = lv == L
+        if lanes[m].sum() > cap:
+            assert (alap[m] == L).all(), L
+    # the schedule is only an order: the plaintext function is unchanged
+    bits = np.random.default_rng(1).integers(0, 2, (3, ni)).astype(np.uint8)
+    want = simulate(ni, net.type, net.in0, net.in1, net.in2, bits)
+    order = np.argsort(lv, kind="stable")
+    inv = np.empty_like(order)
+    inv[order] = np.arange(order.size)
+    remap = lambda w: np.where(w < ni, w, ni + inv[np.maximum(w - ni, 0)])
+    got = simulate(ni, net.type[order], remap(net.in0[order]), np.where(net.in1[order] < 0, -1, remap(net.in1[order])),
+                   np.where(net.in2[order] < 0, -1, remap(net.in2[order])), bits)
+    assert (got[:, ni:][:, inv] == want[:, ni:]).all()
+
+
+def test_capacity_schedule_narrows_vip_levels(tb):
+    """on the VIP-shaped bubble sort, fewer levels exceed one latency-kernel wave (32 bootstraps)"""
+    n = synth.bubble_sort(16, 16)
+    net = tb.Netlist(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"], outputs=n["outputs"])
+    lanes = np.where(net.type == 16, 2, np.where(net.type == 3, 0, 1))
+    over = []
+    for cap in (0, 32):
+        _, _, lv = _sched(net, cap)
+        per = np.bincount(lv, weights=lanes)[1:]
+        over.append(int((per > 32).sum()))
+    assert over[1] < over[0] // 2, over

@@ -30,6 +30,8 @@ def configs():
     yield "cfg4a_mul32x32", synth.array_multiplier(32)
     yield "cfg4b_sort16x16", synth.bubble_sort(16, 16)
     yield "cfg5_mnist_fig4", synth.mnist_fig4()
+    yield "f3_attention_S", synth.attention(4, 32, 4)          # Attention_S shape (hidden 32)
+    yield "f3_attention_L", synth.attention(4, 64, 4)          # Attention_L shape (hidden 64)
 
 
 def main():
