@@ -257,11 +257,12 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
                 x[v] = dcplx{small_to_double((u0 >> shift) & 127u, 64.0), small_to_double((u1 >> shift) & 127u, 64.0)};
             }
             fwd2w(x, S.dslot[jd], t1, t2, t3, tt, 1 + jd);
+            bar_pair(1 + jd);
+            if (tt == 0)   // row jd -> CTA (1-q, h) as soon as this warp pair is done
+                push_peer(rows_dst + (uint32_t)((buf * kL + jd) * 512 * 16), &S.dslot[jd][0], 512 * 16,
+                          rows_mb + (uint32_t)(buf * 8));
         }
         __syncthreads();
-        if (tid == 0)   // our 3 rows -> CTA (1-q, h)
-            push_peer(rows_dst + (uint32_t)(buf * kL * 512 * 16), &S.dslot[0][0], kL * 512 * 16,
-                      rows_mb + (uint32_t)(buf * 8));
         mb_wait(&S.mbar_bk[buf], par);
         // ---- B: out[k] = sum_{r<6} D_r[k] BK_i[r][o][k]; own bloc's rows first, then the other bloc's ----
         dcplx m3[3];
@@ -294,9 +295,9 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
                 stc(&S.oslot[lsw(k)], s);
             }
         }
+        if ((tid & 63) == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // dslot rows sent
         __syncthreads();                                  // bk[buf], rrows[buf] consumed; oslot complete
         if (tid == 0) {
-            asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // dslot readable again (rows sent)
             if (i + 2 < kn) {
                 mb_expect(&S.mbar_rows[buf], kL * 512 * 16);                  // rows of step i + 2
                 issue_bk_l(S, bkf, i + 2, o, buf);
@@ -311,9 +312,10 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
                 S.res[c] = round_mod32(x[v].re) << (16 * h);
                 S.res[c + 512] = round_mod32(x[v].im) << (16 * h);
             }
+            bar_pair(4);
+            if (tid == 0) push_peer(res_dst + (uint32_t)(buf * kN * 4), S.res, kN * 4, res_mb + (uint32_t)(buf * 8));
         }
         __syncthreads();
-        if (tid == 0) push_peer(res_dst + (uint32_t)(buf * kN * 4), S.res, kN * 4, res_mb + (uint32_t)(buf * 8));
         mb_wait(&S.mbar_res[buf], par);
         for (int c = tid; c < kN; c += kLThreads) {       // ACC[q] += lo + 2^16 hi (own half + the sibling's)
             const uint32_t nv = S.acc[c] + S.res[c] + S.rres[buf][c];
