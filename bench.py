@@ -35,6 +35,11 @@ METRIC = "bootstrapped gates/sec (box, device-timed) at 1/2/4/8 B200; % of roofl
 UNIT = "gates/s"
 CMUX_BFLY = 12 * 5 * 1024          # 12 negacyclic NTTs of N = 1024 per CMux step (6 forward + 6 inverse)
 CMUX_MAC = 6 * 6 * 1024            # pointwise 64-bit multiply-accumulates per CMux step
+# FP64 variant (--br-variant 10): FP64-pipe warp instructions per CMux step and lane of the implemented
+# structure (10 transforms of 9 radix-2 stages with 6-DFMA CT / 8-op GS butterflies and constant twiddle
+# factors, 1,536 MAC DFMAs, digit conversions), counted by ncu smsp__inst_executed_pipe_fp64 / (lanes x 630)
+# on a 4,736-lane launch (profiles/r01_ncu_brf_summary.md)
+CMUX_FP64_INSTR = 7032
 N_LWE = 630
 
 
@@ -230,43 +235,55 @@ def main():
         ms = float(t.item())
     value = total * args.steps / (ms / 1e3)
 
-    # roofline of the dominant kernel (blind rotation): the integer-multiply (FMA-heavy) pipe.  Algorithmic
-    # work = IMAD issue slots of the method's modular arithmetic: per CMux step
-    # 61,440 Shoup mulmods x 4 slots (IMAD + IMAD.HI(2) + IMAD) + 36,864 64-bit MACs x 2 (IMAD.WIDE) + 6,144
-    # MAC reductions x 5.  Peak = 148 SMs x 64 IMAD lanes/clk (fma pipe: 16 lanes/clk/SMSP, B300_MICROARCH
-    # "Pipe rates") x the median SM clock sampled during the timed region.
+    # roofline of the dominant kernel (blind rotation).  Integer variants (br6/7/8): the integer-multiply
+    # (FMA-heavy) pipe.  Algorithmic work = IMAD issue slots of the method's modular arithmetic (DESIGN.md
+    # "Roofline"): per CMux step 61,440 Shoup mulmods x 4 slots (IMAD + IMAD.HI(2) + IMAD) + 36,864 64-bit MACs
+    # x 2 (IMAD.WIDE) + 6,144 MAC reductions x 5.  Peak = 148 SMs x 64 IMAD lanes/clk (fma pipe: 16
+    # lanes/clk/SMSP, B300_MICROARCH "Pipe rates") x the median SM clock sampled during the timed region.
+    # FP64 variant (brf): FP64-pipe lane operations of the implemented structure over 148 SMs x 64 FP64
+    # lanes/clk (measured 1.99 warp-instructions/clk/SM by ncu) x the same clock.
     bfly_rate, mac_rate = ctx.microbench()
     g0, g1, _ = tb.parallel.shard(total, world, rank)
     lanes_per_launch = g1 - g0
-    slots_per_bootstrap = N_LWE * (CMUX_BFLY * 4 + CMUX_MAC * 2 + 6 * 1024 * 5)
-    work = slots_per_bootstrap * lanes_per_launch
     br_launch_s = br_ms / max(br_n, 1) / 1e3
-    achieved = work / br_launch_s
     sm_count = torch.cuda.get_device_properties(local).multi_processor_count
     clk_mhz = clocks.get("sm_mhz") or 1965.0
     peak = sm_count * 64 * clk_mhz * 1e6
+    if args.br_variant == 10:
+        per_bootstrap = N_LWE * CMUX_FP64_INSTR * 32
+        unit, pipe = "G FP64-lane-ops/s", "FP64"
+        work_text = "%d FP64 lane-ops = 630 x %d FP64 warp-instructions x 32 lanes" % (per_bootstrap, CMUX_FP64_INSTR)
+    else:
+        per_bootstrap = N_LWE * (CMUX_BFLY * 4 + CMUX_MAC * 2 + 6 * 1024 * 5)
+        unit, pipe = "G IMAD-slots/s", "IMAD"
+        work_text = "%d IMAD slots = 630 x (61,440 mulmod x 4 + 36,864 MAC x 2 + 6,144 reductions x 5)" % per_bootstrap
+    work = per_bootstrap * lanes_per_launch
+    achieved = work / br_launch_s
     bfly_work = N_LWE * (CMUX_BFLY + CMUX_MAC * bfly_rate / mac_rate) * lanes_per_launch
     traffic = None
     prof_path = os.path.join(ROOT, "profiles", "ncu_br_kernel_summary.json")
     if os.path.exists(prof_path):
         try:
             pj = json.load(open(prof_path))
-            if pj.get("lanes") == lanes_per_launch and pj.get("lanes_per_cta") == args.lanes_per_cta:
+            if (pj.get("lanes") == lanes_per_launch and pj.get("lanes_per_cta") == args.lanes_per_cta
+                    and pj.get("br_variant", 6) == args.br_variant):
                 traffic = pj.get("dram_bytes_per_launch")
         except Exception:
             traffic = None
-    roofline = {"bound": "alu", "achieved": achieved / 1e9, "peak": peak / 1e9, "unit": "G IMAD-slots/s",
+    roofline = {"bound": "alu", "achieved": achieved / 1e9, "peak": peak / 1e9, "unit": unit,
                 "frac": achieved / peak, "traffic": traffic,
-                "kernel": "br%d_kernel (blind rotation + extraction)" % args.br_variant, "kernel_ms_per_launch": br_launch_s * 1e3,
+                "kernel": "%s (blind rotation + extraction)" % ("brf_kernel" if args.br_variant == 10
+                                                                 else "br%d_kernel" % args.br_variant),
+                "kernel_ms_per_launch": br_launch_s * 1e3,
                 "kernel_share_of_step": br_ms / ms if ms else None,
                 "ks_kernel_ms_per_launch": ks_ms / max(ks_n, 1),
-                "peak_source": "derived: %d SMs x 64 IMAD lanes/clk x %.0f MHz (median SM clock in the timed region)"
-                               % (sm_count, clk_mhz),
-                "work_per_bootstrap": "%d IMAD slots = 630 x (61,440 mulmod x 4 + 36,864 MAC x 2 + 6,144 reductions x 5)"
-                                      % slots_per_bootstrap,
-                "bootstraps_per_s_at_peak": peak / slots_per_bootstrap,
-                "microbench_crosscheck": {"butterflies_per_s": bfly_rate, "macs_per_s": mac_rate,
-                                          "frac_of_microbench": bfly_work / br_launch_s / bfly_rate}}
+                "peak_source": "derived: %d SMs x 64 %s lanes/clk x %.0f MHz (median SM clock in the timed region)"
+                               % (sm_count, pipe, clk_mhz),
+                "work_per_bootstrap": work_text,
+                "bootstraps_per_s_at_peak": peak / per_bootstrap}
+    if args.br_variant != 10:
+        roofline["microbench_crosscheck"] = {"butterflies_per_s": bfly_rate, "macs_per_s": mac_rate,
+                                             "frac_of_microbench": bfly_work / br_launch_s / bfly_rate}
 
     # narrow-level latency (one gate)
     lat = None
