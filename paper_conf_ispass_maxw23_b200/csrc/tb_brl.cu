@@ -22,6 +22,14 @@ namespace tb {
 
 constexpr int kLThreads = 192;                 // 6 warps: 3 forward transforms x 2 warps; warps 0-1 invert
 
+#ifdef TB_BRL_TRACE   // scratch instrumentation (tools/buildvar.sh WORK name -DTB_BRL_TRACE): clock64 per phase
+__device__ long long g_brl_trace[4][8][16];
+#define BRL_T(p)                                                                                              \
+    if (gl == 0 && tid == 0 && i >= 100 && i < 116) g_brl_trace[rank][p][i - 100] = clock64();
+#else
+#define BRL_T(p)
+#endif
+
 struct __align__(128) BrlSmem {
     double2 bk[2][kRows][512];                 // BK_i, rows 0..5 of output o = 2q + h, by step parity (96 KB)
     double2 dslot[kL][512];                    // own forward rows (bloc q), swizzled positions
@@ -245,6 +253,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
     for (int i = 0; i < kn; i++) {
         const int buf = i & 1;
         const uint32_t par = (uint32_t)((i >> 1) & 1);
+        BRL_T(0)
         {   // ---- A: digit jd of (X^abar - 1) ACC[q], folded, forward transform (warp pair jd) ----
             const uint32_t ab = S.bar[i];
             const uint32_t* win = S.acc + ((tt - (int)ab) & (kTwoN - 1));
@@ -263,7 +272,9 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
                           rows_mb + (uint32_t)(buf * 8));
         }
         __syncthreads();
+        BRL_T(1)
         mb_wait(&S.mbar_bk[buf], par);
+        BRL_T(2)
         // ---- B: out[k] = sum_{r<6} D_r[k] BK_i[r][o][k]; own bloc's rows first, then the other bloc's ----
         dcplx m3[3];
 #pragma unroll
@@ -281,6 +292,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
             m3[e] = s;
         }
         mb_wait(&S.mbar_rows[buf], par);
+        BRL_T(3)
 #pragma unroll
         for (int e = 0; e < 3; e++) {
             const int k = tid + kLThreads * e;
@@ -297,6 +309,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         }
         if ((tid & 63) == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // dslot rows sent
         __syncthreads();                                  // bk[buf], rrows[buf] consumed; oslot complete
+        BRL_T(4)
         if (tid == 0) {
             if (i + 2 < kn) {
                 mb_expect(&S.mbar_rows[buf], kL * 512 * 16);                  // rows of step i + 2
@@ -316,7 +329,9 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
             if (tid == 0) push_peer(res_dst + (uint32_t)(buf * kN * 4), S.res, kN * 4, res_mb + (uint32_t)(buf * 8));
         }
         __syncthreads();
+        BRL_T(5)
         mb_wait(&S.mbar_res[buf], par);
+        BRL_T(6)
         for (int c = tid; c < kN; c += kLThreads) {       // ACC[q] += lo + 2^16 hi (own half + the sibling's)
             const uint32_t nv = S.acc[c] + S.res[c] + S.rres[buf][c];
             S.acc[c] = nv;
@@ -324,6 +339,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
             S.acc[c + 2 * kN] = nv;
         }
         __syncthreads();                                  // rres[buf] consumed
+        BRL_T(7)
         if (tid == 0) {
             asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // res readable again
             if (i + 2 < kn) mb_expect(&S.mbar_res[buf], kN * 4);            // the sibling's half of step i + 2
@@ -371,6 +387,12 @@ int brl_wave_lanes() {
     if (cudaOccupancyMaxActiveClusters(&n, brl_kernel, &cfg) != cudaSuccess) return -1;
     return n;
 }
+
+#ifdef TB_BRL_TRACE
+extern "C" int tb_debug_brl_trace(long long* host) {
+    return cudaMemcpyFromSymbol(host, g_brl_trace, sizeof(g_brl_trace)) == cudaSuccess ? 0 : -1;
+}
+#endif
 
 int launch_brl(const BrArgs& A, const double2* bkf, const double2* twL, cudaStream_t st) {
     const size_t smem = sizeof(BrlSmem);
