@@ -304,16 +304,20 @@ def test_mixed_netlist_with_not_and_mux(tb, ctx, keys):
     assert (O.decrypt_bits(keys, gpu) == plain).all()
 
 
-def test_throughput_level_bench_size_sampled(tb, ctx, keys):
+@pytest.mark.parametrize("variant", [6, 10])
+def test_throughput_level_bench_size_sampled(tb, ctx, keys, variant):
     """BASELINE configs[2] at the bench's per-GPU size (65,536 NAND/XOR gates, one level, the launch
-    configuration bench.py times): all outputs decrypt to the truth; a seeded sample of 48 gates is
-    recomputed by the oracle and compared bit for bit."""
-    import torch
+    configuration bench.py times, default br6 and --br-variant 10): all outputs decrypt to the truth; a
+    seeded sample of 48 gates is recomputed by the oracle and compared bit for bit."""
     G = 65536
     n = synth.independent_level(G, seed=3)
     bits = synth.random_bits(2 * G, 4)
     cts = enc(keys, bits, 5)
-    gpu = run_netlist_gpu(tb, ctx, n, cts)
+    ctx.set_br_variant(variant)
+    try:
+        gpu = run_netlist_gpu(tb, ctx, n, cts)
+    finally:
+        ctx.set_br_variant(6)
     out = gpu[2 * G:]
     truth = ((n["type"].astype(np.int64) >> (2 * bits[0::2].astype(np.int64) + bits[1::2])) & 1).astype(np.uint8)
     assert (O.decrypt_bits(keys, out) == truth).all()
