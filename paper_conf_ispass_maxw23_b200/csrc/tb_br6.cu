@@ -85,7 +85,7 @@ __global__ void __launch_bounds__(192 * G, (G <= 2 ? 2 : 1)) br6_kernel(BrArgs A
                 const uint32_t mm = (c - ab) & (kTwoN - 1);           // X^ab ACC: coefficient c
                 const uint32_t src = acc[mm & (kN - 1)];
                 const uint32_t rot = mm < (uint32_t)kN ? src : 0u - src;
-                const uint32_t u = rot - acc[c] + kDecompOffset;      // (X^ab - 1) ACC + offset
+                const uint32_t u = rot - acc[c] + c_misc[3];          // (X^ab - 1) ACC + offset (misc[3])
                 x[j] = ((u >> shift) & 127u) + (kP - 64u);             // digit in [-64, 63], as mod p
             }
             uint32_t* slot = S.slot[g][w6];
@@ -141,7 +141,7 @@ __global__ void __launch_bounds__(192 * G, (G <= 2 ? 2 : 1)) br6_kernel(BrArgs A
                 uint32_t* acc = S.acc[g][q];
 #pragma unroll
                 for (int j = 0; j < 32; j++)
-                    acc[lane + 32 * j] += x[j] + p1[kPadRow * j + lane] + p2[kPadRow * j + lane];
+                    acc[lane + 32 * j] = add_alu(acc[lane + 32 * j] + x[j] + p1[kPadRow * j + lane], p2[kPadRow * j + lane]);
             }
         }
         __syncthreads();

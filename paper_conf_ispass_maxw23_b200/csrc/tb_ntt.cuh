@@ -18,8 +18,17 @@ namespace tb {
 // warp-uniform twiddles of stages 0-4 (k = 1..31) and their Shoup companions floor(w 2^32 / p).
 // (The library is one translation unit, tb_lib.cu, so these are defined here.)
 __constant__ uint32_t c_fw[32], c_fwp[32], c_iw[32], c_iwp[32];
-// misc constants: [0] = 2^32 mod p, [1] = Shoup(2^32 mod p)
+// misc constants: [0] = 2^32 mod p, [1] = Shoup(2^32 mod p), [2] = 2p (as a constant-bank operand, below),
+// [3] = the gadget decomposition offset
 __constant__ uint32_t c_misc[4];
+// Always 0.  Butterfly sums are written as x + y + c_zero: a three-input add can only be an ALU IADD3, while
+// a plain x + y is often emitted as IMAD.IADD on the FMA pipe -- the pipe the Shoup products saturate
+// (measured: ~150 of the ~640 butterfly adds per thread and transform pair went to IMAD.IADD, 12 % more
+// FMA-pipe cycles).
+__constant__ uint32_t c_zero;
+__device__ __forceinline__ uint32_t add_alu(uint32_t a, uint32_t b) { return a + b + c_zero; }
+// a - b + 2p with 2p from the constant bank: one IADD3 (with the immediate, ptxas splits off a - b as IMAD.IADD)
+__device__ __forceinline__ uint32_t sub_alu(uint32_t a, uint32_t b) { return a - b + c_misc[2]; }
 
 __device__ __forceinline__ uint32_t shoup_mul(uint32_t y, uint32_t w, uint32_t wp) {
     // y * w mod p in [0, 2p) for any y < 2^32 (Shoup)
@@ -40,13 +49,13 @@ __device__ __forceinline__ int sidx(int row, int col) {
 __device__ __forceinline__ void ct_bfly(uint32_t& x, uint32_t& y, uint32_t w, uint32_t wp) {
     const uint32_t X = red_2p(x);
     const uint32_t T = shoup_mul(y, w, wp);
-    x = X + T;
-    y = X - T + kTwoP;
+    x = add_alu(X, T);
+    y = sub_alu(X, T);
 }
 // GS butterfly, inputs and outputs in [0, 2p)
 __device__ __forceinline__ void gs_bfly(uint32_t& x, uint32_t& y, uint32_t w, uint32_t wp) {
-    const uint32_t S = red_2p(x + y);
-    const uint32_t D = x - y + kTwoP;
+    const uint32_t S = red_2p(add_alu(x, y));
+    const uint32_t D = sub_alu(x, y);
     x = S;
     y = shoup_mul(D, w, wp);
 }

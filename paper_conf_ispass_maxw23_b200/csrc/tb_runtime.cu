@@ -208,6 +208,8 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
     }
     misc[0] = (uint32_t)((1ull << 32) % kP);
     misc[1] = shoup_of(misc[0]);
+    misc[2] = kTwoP;
+    misc[3] = kDecompOffset;
     std::vector<uint2> tf(31 * 32), ti(31 * 32);
     for (int s = 5; s < 10; s++)
         for (int bj = 0; bj < (1 << (s - 5)); bj++)
