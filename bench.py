@@ -161,9 +161,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--gates-per-gpu", type=int, default=65536)
     ap.add_argument("--lanes-per-cta", type=int, default=2)
-    ap.add_argument("--br-variant", type=int, default=6, choices=[6, 7, 8, 10, 12])
-    ap.add_argument("--mix", default="300,118784,1",
-                    help="variant 12: FP64 share (permille), br6 shared-memory request (bytes), brf lanes/CTA")
+    ap.add_argument("--br-variant", type=int, default=6, choices=[6, 7, 8, 10])
     ap.add_argument("--ks-tile", type=int, default=8, choices=[8, 16, 32])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -196,7 +194,6 @@ def main():
     ctx = tb.Context(local)
     ctx.set_lanes_per_cta(args.lanes_per_cta)
     ctx.set_br_variant(args.br_variant)
-    ctx.set_mix(*[int(x) for x in args.mix.split(",")])
     ctx.set_ks_tile(args.ks_tile)
     ctx.load_keys(synth.random_words(tb.BK_WORDS, 11), synth.random_words(tb.KSK_WORDS, 12))
     n = synth.independent_level(total, seed=13)

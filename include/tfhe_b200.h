@@ -172,12 +172,6 @@ int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
  * (2 lanes/CTA, 1 CTA/SM, each 144 KB BK step TMA-bulk-copied into shared memory one step ahead).  Both are
  * bit-identical; see DESIGN.md "Kernels". */
 int tb_set_br_variant(tb_ctx* ctx, int variant);
-/* Variant 12 ("mixed"): each throughput launch is split, lanes [0, n6) on br6_kernel<2> (integer NTT, IMAD
- * pipe) and the rest on brf_kernel<fp_lanes_per_cta> (FP64 FFT, FP64 pipe), launched concurrently so that an
- * SM runs one of each (br6 on a high-priority internal stream with its shared-memory request padded to
- * `br6_smem_bytes`).  `fp_permille` = share of lanes given to brf (0..1000).  Outputs are bit-identical to
- * every other variant.  Invalid values: TB_EINVAL.  Defaults: 300, 118784, 1. */
-int tb_set_mix(tb_ctx* ctx, int fp_permille, int br6_smem_bytes, int fp_lanes_per_cta);
 /* Latency mode for narrow levels: a launch with <= `lanes` bootstraps runs a latency-mode kernel (below)
  * instead of the throughput kernel.  Default = the device's SM count; 0 disables. */
 int tb_set_narrow_lanes(tb_ctx* ctx, int64_t lanes);

@@ -119,13 +119,8 @@ class Context:
         _native.check(_native.lib().tb_set_lanes_per_cta(self._h, lanes))
 
     def set_br_variant(self, variant: int):
-        """6 = br6_kernel (default), 7 = br7_kernel (TMA-staged BK), 8 = br8_kernel, 10 = brf_kernel (FP64),
-        12 = br6 + brf co-resident (see set_mix); bit-identical outputs."""
+        """6 = br6_kernel (default), 7 = br7_kernel (TMA-staged BK); bit-identical outputs."""
         _native.check(_native.lib().tb_set_br_variant(self._h, variant))
-
-    def set_mix(self, fp_permille: int = 300, br6_smem_bytes: int = 116 * 1024, fp_lanes_per_cta: int = 1):
-        """variant 12: share of lanes on the FP64 kernel, br6 shared-memory request, brf lanes per CTA"""
-        _native.check(_native.lib().tb_set_mix(self._h, fp_permille, br6_smem_bytes, fp_lanes_per_cta))
 
     def set_narrow_lanes(self, lanes: int):
         """levels with <= lanes bootstraps run in latency mode (see set_narrow_kernel); 0 disables"""

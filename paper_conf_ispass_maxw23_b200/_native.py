@@ -90,7 +90,6 @@ SIGNATURES = {
     "tb_fft_muladd6": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
     "tb_set_lanes_per_cta": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_set_br_variant": (ctypes.c_int, [_vp, ctypes.c_int]),
-    "tb_set_mix": (ctypes.c_int, [_vp, ctypes.c_int, ctypes.c_int, ctypes.c_int]),
     "tb_set_ks_tile": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_set_narrow_lanes": (ctypes.c_int, [_vp, _i64]),
     "tb_set_narrow_kernel": (ctypes.c_int, [_vp, ctypes.c_int]),

@@ -163,14 +163,13 @@ __global__ void __launch_bounds__(192 * G, (G <= 2 ? 2 : 1)) br6_kernel(BrArgs A
 }
 
 template <int G>
-static int launch_br6_g(const BrArgs& A, cudaStream_t st, size_t smem_min) {
-    // smem_min > sizeof pads the CTA's shared-memory request (co-residence control of the mixed variant)
-    const size_t smem = sizeof(Br6Smem<G>) > smem_min ? sizeof(Br6Smem<G>) : smem_min;
-    static size_t attr = 0;
-    if (smem > attr) {
+static int launch_br6_g(const BrArgs& A, cudaStream_t st) {
+    const size_t smem = sizeof(Br6Smem<G>);
+    static bool attr = false;
+    if (!attr) {
         if (cudaFuncSetAttribute(br6_kernel<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
             return -1;
-        attr = smem;
+        attr = true;
     }
     const int blocks = (A.nlanes + G - 1) / G;
     if (blocks == 0) return 0;
@@ -178,12 +177,12 @@ static int launch_br6_g(const BrArgs& A, cudaStream_t st, size_t smem_min) {
     return 0;
 }
 
-int launch_br6(const BrArgs& A, int G, cudaStream_t st, size_t smem_min) {
+int launch_br6(const BrArgs& A, int G, cudaStream_t st) {
     switch (G) {
-        case 1: return launch_br6_g<1>(A, st, smem_min);
-        case 2: return launch_br6_g<2>(A, st, smem_min);
-        case 3: return launch_br6_g<3>(A, st, smem_min);
-        case 4: return launch_br6_g<4>(A, st, smem_min);
+        case 1: return launch_br6_g<1>(A, st);
+        case 2: return launch_br6_g<2>(A, st);
+        case 3: return launch_br6_g<3>(A, st);
+        case 4: return launch_br6_g<4>(A, st);
         default: return -2;
     }
 }

@@ -35,7 +35,7 @@ struct KsArgs {
     int64_t not_stride;
 };
 
-int launch_br6(const BrArgs& A, int G, cudaStream_t st, size_t smem_min = 0);
+int launch_br6(const BrArgs& A, int G, cudaStream_t st);
 int launch_br7(const BrArgs& A, int G, cudaStream_t st);
 int launch_br8(const BrArgs& A, cudaStream_t st);
 int launch_br9(const BrArgs& A, cudaStream_t st);

@@ -69,12 +69,6 @@ struct tb_ctx {
     int64_t level_capacity = -1;            // netlist upload: re-levelise to <= this many lanes per level where
                                             // slack allows (0 = Algorithm 1 as is, -1 = auto: brl_wave)
     cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
-    // variant 12 (mixed): br6 and brf co-resident on every SM (IMAD pipe + FP64 pipe)
-    int mix_fp_permille = 300;              // share of a launch's lanes given to brf<1>
-    int mix_br6_smem = 116 * 1024;          // br6<2> shared-memory request (> half an SM: one br6 CTA per SM)
-    int mix_fp_G = 1;                       // brf lanes per CTA in the mix
-    cudaStream_t side = nullptr;            // high-priority stream the mix launches br6 on
-    cudaEvent_t fork = nullptr, join = nullptr;
     uint2* twF = nullptr;                   // [31][32]
     uint2* twI = nullptr;
     double2* fftB = nullptr;                // FP64 FFT per-lane twiddles: stages 5-8 [15][32], stage 9 [8][32]
@@ -285,9 +279,6 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
     cudaFree(c->ks_scratch);
     for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
     if (c->own) cudaStreamDestroy(c->own);
-    if (c->side) cudaStreamDestroy(c->side);
-    if (c->fork) cudaEventDestroy(c->fork);
-    if (c->join) cudaEventDestroy(c->join);
     delete c;
     return TB_OK;
 }
@@ -299,8 +290,8 @@ extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
 }
 
 extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
-    if (!c || !(variant == 6 || variant == 7 || variant == 8 || variant == 10 || variant == 12))
-        return fail(TB_EINVAL, "blind-rotation variant must be 6, 7, 8, 10 or 12");
+    if (!c || !(variant == 6 || variant == 7 || variant == 8 || variant == 10))
+        return fail(TB_EINVAL, "blind-rotation variant must be 6, 7, 8 or 10");
     c->variant = variant;
     return TB_OK;
 }
@@ -408,47 +399,6 @@ static int check_ready(tb_ctx* c) {
     return TB_OK;
 }
 
-extern "C" int tb_set_mix(tb_ctx* c, int fp_permille, int br6_smem_bytes, int fp_lanes_per_cta) {
-    if (!c || fp_permille < 0 || fp_permille > 1000 || br6_smem_bytes < 0 || br6_smem_bytes > 227 * 1024 ||
-        fp_lanes_per_cta < 1 || fp_lanes_per_cta > 3)
-        return fail(TB_EINVAL, "mix: permille 0..1000, br6 shared memory 0..232448 bytes, FP64 lanes per CTA 1..3");
-    c->mix_fp_permille = fp_permille;
-    c->mix_br6_smem = br6_smem_bytes;
-    c->mix_fp_G = fp_lanes_per_cta;
-    return TB_OK;
-}
-
-// Variant 12: split the launch's lanes between br6<2> (integer NTT, IMAD pipe) and brf (FP64 FFT, FP64 pipe)
-// and run both at once, br6 on a high-priority stream with its shared-memory request padded so that an SM
-// holds one br6 CTA and the FP64 CTA(s) beside it.  Both kernels are bit-identical, so the split is free.
-static int launch_mixed(tb_ctx* c, const BrArgs& A, cudaStream_t st) {
-    if (!c->side) {
-        int lo = 0, hi = 0;
-        cudaDeviceGetStreamPriorityRange(&lo, &hi);
-        if (cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, hi) != cudaSuccess ||
-            cudaEventCreateWithFlags(&c->fork, cudaEventDisableTiming) != cudaSuccess ||
-            cudaEventCreateWithFlags(&c->join, cudaEventDisableTiming) != cudaSuccess)
-            return -1;
-    }
-    int64_t nf = (int64_t)A.nlanes * c->mix_fp_permille / 1000;
-    int64_t n6 = A.nlanes - nf;
-    n6 -= n6 & 1;                       // br6<2> CTAs stay full
-    nf = A.nlanes - n6;
-    BrArgs A6 = A, Af = A;
-    A6.nlanes = (int32_t)n6;
-    Af.lanes = A.lanes + n6;
-    Af.out = A.out + n6 * A.out_stride;
-    Af.nlanes = (int32_t)nf;
-    int rc = 0;
-    if (cudaEventRecord(c->fork, st) != cudaSuccess || cudaStreamWaitEvent(c->side, c->fork, 0) != cudaSuccess)
-        return -1;
-    if (n6 > 0) rc = launch_br6(A6, 2, c->side, (size_t)c->mix_br6_smem);
-    if (!rc && nf > 0) rc = launch_brf(Af, c->mix_fp_G, c->bkf, c->fftB, c->fftC, st);
-    if (cudaEventRecord(c->join, c->side) != cudaSuccess || cudaStreamWaitEvent(st, c->join, 0) != cudaSuccess)
-        return -1;
-    return rc;
-}
-
 static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint32_t* s2, int64_t sstride,
                   const LaneDesc* lanes, int64_t nlanes, uint32_t* out, int64_t ostride, cudaStream_t st) {
     if (nlanes <= 0) return TB_OK;
@@ -473,8 +423,6 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
         rc = launch_brf(A, std::min(std::max(c->lanes_per_cta, 1), 3), c->bkf, c->fftB, c->fftC, st);
     else if (c->variant == 8)
         rc = launch_br8(A, st);
-    else if (c->variant == 12)
-        rc = launch_mixed(c, A, st);
     else
         rc = launch_br6(A, c->lanes_per_cta, st);
     prof_end(c, slot, st);
