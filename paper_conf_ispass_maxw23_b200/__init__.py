@@ -226,18 +226,73 @@ class Context:
         _native.check(_native.lib().tb_run_level(self._h, dnet._h, level, g0, g1, _ptr(wires), wires.stride(0),
                                                  _stream_handle(stream)))
 
-    def run_netlist(self, dnet: DevNetlist, wires: torch.Tensor, group=None, stream=None):
+    def run_netlist(self, dnet: DevNetlist, wires: torch.Tensor, group=None, stream=None, exchange: str = "fused"):
         """Evaluate every level.  Without a process group: one device (tb_run_netlist).  With one: each
-        level's gates are split into R contiguous chunks, rank r evaluates chunk r, and the output rows are
-        all-gathered in place over NCCL before the next level."""
+        level's gates are split into R contiguous chunks and rank r evaluates chunk r; the level's output rows
+        reach every rank either through the key-switch kernels' own stores into the peers' wire arrays
+        (exchange="fused": CUDA-IPC peer memory, tb_set_peer_wires, then a barrier) or through an in-place
+        all-gather over the process group (exchange="allgather").  DESIGN.md "Multi-GPU"."""
+        _check_dev(wires, self.device, "wires")
         if group is None:
-            _check_dev(wires, self.device, "wires")
             _native.check(_native.lib().tb_run_netlist(self._h, dnet._h, _ptr(wires), wires.stride(0),
                                                        _stream_handle(stream)))
             return
-        _check_dev(wires, self.device, "wires")
-        parallel.level_loop([(row0, ng) for row0, ng, _, _ in dnet.levels], wires,
-                            lambda L, g0, g1: self.run_level(dnet, L, g0, g1, wires, stream), group)
+        if exchange not in ("fused", "allgather"):
+            raise ValueError("exchange must be 'fused' or 'allgather'")
+        levels = [(row0, ng) for row0, ng, _, _ in dnet.levels]
+        run = lambda L, g0, g1: self.run_level(dnet, L, g0, g1, wires, stream)   # noqa: E731
+        if exchange == "fused":
+            self.attach_peers(wires, group)
+            parallel.level_loop(levels, wires, run, group, fused=True)
+        else:
+            parallel.level_loop(levels, wires, run, group)
+
+    # ---- fused all-gather: the other ranks' wire arrays mapped into this process (CUDA IPC) ----
+    def attach_peers(self, wires: torch.Tensor, group):
+        """Map every other rank's `wires` (same shape and stride) into this process and make tb_run_level's
+        key-switch kernels store each output row into all of them (tb_set_peer_wires).  Collective over
+        `group`; a no-op when this exact tensor is already attached."""
+        import torch.distributed as dist
+        key = (wires.data_ptr(), tuple(wires.shape), wires.stride(0))
+        if getattr(self, "_peer_key", None) == key:
+            return
+        self.detach_peers()
+        R, r = dist.get_world_size(group), dist.get_rank(group)
+        h = (ctypes.c_ubyte * 64)()
+        off = ctypes.c_int64()
+        _native.check(_native.lib().tb_ipc_export(_ptr(wires), h, ctypes.byref(off)))
+        mine = (bytes(h), off.value, tuple(wires.shape), wires.stride(0))
+        allh = [None] * R
+        dist.all_gather_object(allh, mine, group=group)
+        ptrs, bases = [], []
+        try:
+            for k, (hb, o, shape, stride) in enumerate(allh):
+                if k == r:
+                    continue
+                if shape != tuple(wires.shape) or stride != wires.stride(0):
+                    raise ValueError("rank %d's wire array has shape %s / stride %d, not %s / %d"
+                                     % (k, shape, stride, tuple(wires.shape), wires.stride(0)))
+                p, b = ctypes.c_void_p(), ctypes.c_void_p()
+                buf = (ctypes.c_ubyte * 64).from_buffer_copy(hb)
+                _native.check(_native.lib().tb_ipc_import(self._h, buf, o, ctypes.byref(p), ctypes.byref(b)))
+                ptrs.append(p.value)
+                bases.append(b.value)
+            arr = (ctypes.c_void_p * max(len(ptrs), 1))(*ptrs)
+            _native.check(_native.lib().tb_set_peer_wires(self._h, arr, len(ptrs)))
+        except Exception:
+            for b in bases:
+                _native.lib().tb_ipc_close(self._h, ctypes.c_void_p(b))
+            raise
+        self._peer_bases, self._peer_key = bases, key
+
+    def detach_peers(self):
+        """Stop storing into peer arrays and unmap them."""
+        bases = getattr(self, "_peer_bases", [])
+        if getattr(self, "_h", None):
+            _native.check(_native.lib().tb_set_peer_wires(self._h, None, 0))
+            for b in bases:
+                _native.lib().tb_ipc_close(self._h, ctypes.c_void_p(b))
+        self._peer_bases, self._peer_key = [], None
 
     def run_netlist_host(self, dnet: DevNetlist, inputs: np.ndarray, output_wires) -> np.ndarray:
         """End-to-end through HOST buffers (tb_run_netlist_host): input ciphertexts [n_inputs, >=631] u32 ->
@@ -271,6 +326,10 @@ class Context:
 
     def close(self):
         if getattr(self, "_h", None):
+            try:
+                self.detach_peers()
+            except Exception:
+                pass
             _native.lib().tb_ctx_destroy(self._h)
             self._h = None
 

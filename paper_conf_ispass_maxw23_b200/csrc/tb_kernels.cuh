@@ -33,6 +33,10 @@ struct KsArgs {
     int64_t out_stride;
     const uint32_t* not_src;    // NOT input rows
     int64_t not_stride;
+    // fused all-gather (multi-GPU level loop): every output row is also stored, at the same row offset, into the
+    // npeers other ranks' wire arrays (peer memory mapped into this process); 0 = own array only
+    uint32_t* const* peers;     // device array [npeers] of peer wire bases (same stride as out)
+    int32_t npeers;
 };
 
 int launch_br6(const BrArgs& A, int G, cudaStream_t st);

@@ -85,12 +85,20 @@ __global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A) {
         for (int g = 0; g < T; g++) {
             const int gi = g0 + g;
             if (gi < A.ngates) {
-                uint32_t* o = A.out + (int64_t)A.gates[gi].out_row * A.out_stride;
+                const int64_t off = (int64_t)A.gates[gi].out_row * A.out_stride;
+                uint32_t* o = A.out + off;
 #pragma unroll
                 for (int q = 0; q < 4; q++)
                     if (k0 + q <= kn) o[k0 + q] = acc[g][q];
+                for (int p = 0; p < A.npeers; p++) {   // fused all-gather: the same row into every peer's array
+                    uint32_t* po = A.peers[p] + off;
+#pragma unroll
+                    for (int q = 0; q < 4; q++)
+                        if (k0 + q <= kn) po[k0 + q] = acc[g][q];
+                }
             }
         }
+        if (A.npeers) __threadfence_system();
     }
 }
 
@@ -157,13 +165,16 @@ __global__ void __launch_bounds__(kKsThreads) ks_split_kernel(KsArgs A, uint32_t
 
 __global__ void __launch_bounds__(kKsThreads) ks_reduce_kernel(KsArgs A, const uint32_t* __restrict__ partial) {
     const int gi = blockIdx.x;
-    uint32_t* o = A.out + (int64_t)A.gates[gi].out_row * A.out_stride;
+    const int64_t off = (int64_t)A.gates[gi].out_row * A.out_stride;
+    uint32_t* o = A.out + off;
     for (int k = threadIdx.x; k <= kn; k += kKsThreads) {
         uint32_t v = 0u;
 #pragma unroll
         for (int s = 0; s < kKsSplit; s++) v += partial[((size_t)gi * kKsSplit + s) * kKsRow + k];
         o[k] = v;
+        for (int p = 0; p < A.npeers; p++) A.peers[p][off + k] = v;   // fused all-gather
     }
+    if (A.npeers) __threadfence_system();
 }
 
 int launch_ks_split(const KsArgs& A, uint32_t* partial, cudaStream_t st) {

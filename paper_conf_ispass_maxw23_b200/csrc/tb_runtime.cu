@@ -2,6 +2,7 @@
 // levelisation and the level executor.  Host-side C++17; every arithmetic step of a gate runs in the
 // kernels of tb_bootstrap.cu / tb_keyswitch.cu.  There is no CPU fallback: without a usable sm_100 device
 // every entry point fails with an error status.
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -91,6 +92,8 @@ struct tb_ctx {
     size_t hwires_words = 0;
     int64_t* hidx = nullptr;                // tb_run_netlist_host gather rows
     int64_t hidx_n = 0;
+    uint32_t** peers = nullptr;             // fused all-gather: device array of the other ranks' wire bases
+    int32_t npeers = 0;
     uint32_t* ks_scratch = nullptr;         // split key-switch partial sums (narrow levels)
     size_t ks_scratch_words = 0;
     // per-kernel event timing (tb_profile_*)
@@ -277,6 +280,7 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
     cudaFree(c->hwires);
     cudaFree(c->hidx);
     cudaFree(c->ks_scratch);
+    cudaFree(c->peers);
     for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
     if (c->own) cudaStreamDestroy(c->own);
     delete c;
@@ -433,12 +437,14 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
 }
 static int run_ks(tb_ctx* c, const uint32_t* lanes, int64_t lane_base, int64_t lane_stride, const GateDesc* gates,
                   int64_t ngates, uint32_t* out, int64_t ostride, const uint32_t* not_src, int64_t not_stride,
-                  cudaStream_t st) {
+                  cudaStream_t st, uint32_t* const* peers = nullptr, int32_t npeers = 0) {
     if (ngates <= 0) return TB_OK;
     KsArgs A;
     A.lanes = lanes; A.lane_base = (int32_t)lane_base; A.lane_stride = lane_stride; A.gates = gates;
     A.ngates = (int32_t)ngates; A.ksk = c->ksk; A.out = out; A.out_stride = ostride; A.not_src = not_src;
     A.not_stride = not_stride;
+    A.peers = peers;
+    A.npeers = npeers;
     const bool split = c->narrow_lanes > 0 && ngates <= c->narrow_lanes;   // narrow level: split each gate's KS
     if (split && c->ks_scratch_words < ks_split_scratch_words(ngates)) {
         cudaFree(c->ks_scratch);
@@ -863,8 +869,80 @@ extern "C" int tb_run_level(tb_ctx* c, const tb_dev_netlist* d, int64_t level, i
     if ((rc = grow_lanes(c, std::max<int64_t>(l1 - l0, 1)))) return rc;
     cudaStream_t st = (cudaStream_t)stream;
     if ((rc = run_br(c, wires, wires, wires, stride, d->ldesc + l0, l1 - l0, c->lanebuf, kLaneStride, st))) return rc;
-    return run_ks(c, c->lanebuf, l0, kLaneStride, d->gdesc + G0, G1 - G0, wires, stride, wires, stride, st);
+    return run_ks(c, c->lanebuf, l0, kLaneStride, d->gdesc + G0, G1 - G0, wires, stride, wires, stride, st,
+                  c->peers, c->npeers);
 }
+
+// ------------------------------------------------------------------------------------------ fused all-gather
+// The multi-GPU level loop's exchange step: instead of a per-level NCCL all-gather, the
+// key-switch kernels store every output row into all ranks' wire arrays over NVLink (peer memory opened with
+// CUDA IPC), so the transfer overlaps the key switch tile by tile; the loop then only needs a barrier.
+extern "C" int tb_set_peer_wires(tb_ctx* c, uint32_t* const* peer_wires, int n) {
+    if (!c || n < 0 || (n > 0 && !peer_wires)) return fail(TB_EINVAL, "bad peer list");
+    for (int k = 0; k < n; k++)
+        if (!peer_wires[k]) return fail(TB_EINVAL, "null peer wire array");
+    TB_CUDA(cudaSetDevice(c->device));
+    cudaFree(c->peers);
+    c->peers = nullptr;
+    c->npeers = 0;
+    if (n == 0) return TB_OK;
+    TB_CUDA(cudaMalloc(&c->peers, (size_t)n * sizeof(uint32_t*)));
+    TB_CUDA(cudaMemcpy(c->peers, peer_wires, (size_t)n * sizeof(uint32_t*), cudaMemcpyHostToDevice));
+    c->npeers = n;
+    return TB_OK;
+}
+
+// base of the device allocation holding p (driver cuMemGetAddressRange through the runtime's entry-point query,
+// so the library does not link libcuda)
+static int alloc_base(const void* p, void** base) {
+    using Fn = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
+    static Fn fn = nullptr;
+    if (!fn) {
+        void* f = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) != cudaSuccess || !f ||
+            q != cudaDriverEntryPointSuccess)
+            return -1;
+        fn = (Fn)f;
+    }
+    CUdeviceptr b = 0;
+    size_t size = 0;
+    if (fn(&b, &size, (CUdeviceptr)p) != CUDA_SUCCESS) return -1;
+    *base = (void*)b;
+    return 0;
+}
+
+extern "C" int tb_ipc_export(const void* dev_ptr, unsigned char* handle, int64_t* offset) {
+    if (!dev_ptr || !handle || !offset) return fail(TB_EINVAL, "null argument");
+    void* base = nullptr;
+    if (alloc_base(dev_ptr, &base)) return fail(TB_ECUDA, "device allocation base lookup failed");
+    cudaIpcMemHandle_t h;
+    TB_CUDA(cudaIpcGetMemHandle(&h, base));
+    static_assert(sizeof(h) == TB_IPC_HANDLE_BYTES, "IPC handle size");
+    memcpy(handle, &h, sizeof(h));
+    *offset = (int64_t)((const char*)dev_ptr - (const char*)base);
+    return TB_OK;
+}
+
+extern "C" int tb_ipc_import(tb_ctx* c, const unsigned char* handle, int64_t offset, void** dev_ptr, void** base) {
+    if (!c || !handle || !dev_ptr || !base || offset < 0) return fail(TB_EINVAL, "bad argument");
+    TB_CUDA(cudaSetDevice(c->device));
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle, sizeof(h));
+    void* b = nullptr;
+    TB_CUDA(cudaIpcOpenMemHandle(&b, h, cudaIpcMemLazyEnablePeerAccess));
+    *base = b;
+    *dev_ptr = (char*)b + offset;
+    return TB_OK;
+}
+
+extern "C" int tb_ipc_close(tb_ctx* c, void* base) {
+    if (!c || !base) return fail(TB_EINVAL, "null argument");
+    TB_CUDA(cudaSetDevice(c->device));
+    TB_CUDA(cudaIpcCloseMemHandle(base));
+    return TB_OK;
+}
+
 
 extern "C" int tb_run_netlist(tb_ctx* c, const tb_dev_netlist* d, uint32_t* wires, int64_t stride, tb_stream stream) {
     if (!d) return fail(TB_EINVAL, "null netlist");

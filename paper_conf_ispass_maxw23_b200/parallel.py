@@ -4,7 +4,9 @@ The paper's backend runs Algorithm 1 and submits every gate of `C - finished` as
 (P:198-203); its only communication is shipping 2.46 KB ciphertexts.  On one 8xB200 box
 the same structure becomes: every rank holds the keys (P:239's broadcast, done once at load) and the whole wire
 array; each level's gates are split into R contiguous chunks, rank r evaluates chunk r, and one in-place
-all-gather over NCCL/NVLink completes the level's output rows on every rank before the next level starts.
+all-gather over NCCL/NVLink completes the level's output rows on every rank before the next level starts --
+or, fused, the key-switch kernels store each output row straight into every rank's wire array over NVLink
+(peer memory) and the level ends with a barrier.
 Output bytes are independent of R (integer-exact kernels), so the result is byte-identical for R = 1..8.
 """
 from __future__ import annotations
@@ -27,19 +29,37 @@ def slack_rows(levels, n_rows: int, world: int) -> int:
     return need
 
 
-def level_loop(levels, wires, run_level, group=None):
+def barrier(group, device=None):
+    """Stream-ordered barrier across ranks: with NCCL a one-element all-reduce on the current stream (every
+    rank's earlier kernels on that stream are done before any rank passes it); otherwise synchronise the
+    device and take the backend's barrier."""
+    import torch
+    import torch.distributed as dist
+    if dist.get_backend(group) == "nccl":
+        dist.all_reduce(torch.zeros(1, device=device), group=group)
+    else:
+        if device is not None and torch.device(device).type == "cuda":
+            torch.cuda.synchronize(device)
+        dist.barrier(group=group)
+
+
+def level_loop(levels, wires, run_level, group=None, fused=False):
     """levels: [(row0, n_gates)] for levels 1..L; run_level(level, g0, g1) evaluates a gate range of a level
-    into `wires` (a [rows, stride] tensor); with a process group of R > 1 ranks the level's output rows are
-    all-gathered in place after each level."""
+    into `wires` (a [rows, stride] tensor).  With a process group of R > 1 ranks every level's output rows must
+    reach all ranks before the next level: fused=True means run_level's kernels already stored them into every
+    rank's array (fused all-gather), so only a barrier is taken; otherwise they are all-gathered in place."""
     import torch.distributed as dist
     R = dist.get_world_size(group) if group is not None else 1
     r = dist.get_rank(group) if group is not None else 0
     for L, (row0, ng) in enumerate(levels, start=1):
         g0, g1, chunk = shard(ng, R, r)
-        if R > 1 and row0 + R * chunk > wires.shape[0]:
+        if R > 1 and not fused and row0 + R * chunk > wires.shape[0]:
             raise ValueError("wire array needs slack rows for the padded all-gather (see slack_rows)")
         if g1 > g0:
             run_level(L, g0, g1)
         if R > 1 and chunk:
-            dist.all_gather_into_tensor(wires[row0:row0 + R * chunk], wires[row0 + r * chunk:row0 + (r + 1) * chunk],
-                                        group=group)
+            if fused:
+                barrier(group, wires.device)
+            else:
+                dist.all_gather_into_tensor(wires[row0:row0 + R * chunk],
+                                            wires[row0 + r * chunk:row0 + (r + 1) * chunk], group=group)

@@ -29,7 +29,7 @@ def _netlist(seed):
     return random_dag(seed, n_inputs=7, n_gates=90)
 
 
-def _worker(rank, world, port, seed, q):
+def _worker(rank, world, port, seed, q, shared=None):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -42,7 +42,8 @@ def _worker(rank, world, port, seed, q):
         order = np.argsort(rows[n_in:])                  # level-sorted position -> original gate index
         bits = np.random.default_rng(seed).integers(0, 2, n_in).astype(np.int32)
         slack = parallel.slack_rows(levels, net.n_wires, world)
-        wires = torch.full((net.n_wires + slack, 3), -1, dtype=torch.int32)
+        fused = shared is not None                    # every rank's array in shared memory: the "peer" stores
+        wires = shared[rank] if fused else torch.full((net.n_wires + slack, 3), -1, dtype=torch.int32)
         wires[:n_in, 0] = torch.from_numpy(bits)
         calls = []
 
@@ -54,10 +55,12 @@ def _worker(rank, world, port, seed, q):
                 x = int(wires[rows[a[g]], 0])
                 y = int(wires[rows[b[g]], 0]) if t[g] != 3 else 0
                 z = int(wires[rows[c[g]], 0]) if t[g] == 16 else 0
-                wires[n_in + k, 0] = int(gate_bits(int(t[g]), x, y, z))
-                wires[n_in + k, 1] = rank                  # who computed it
+                v = int(gate_bits(int(t[g]), x, y, z))
+                for dst in (shared if fused else [wires]):  # fused: the row goes to every rank's array
+                    dst[n_in + k, 0] = v
+                    dst[n_in + k, 1] = rank                # who computed it
 
-        parallel.level_loop(levels, wires, run_level, group=dist.group.WORLD)
+        parallel.level_loop(levels, wires, run_level, group=dist.group.WORLD, fused=fused)
         q.put((rank, wires[:net.n_wires].numpy().copy(), calls, rows))
     finally:
         dist.destroy_process_group()
@@ -88,6 +91,34 @@ def test_level_loop_all_gather_matches_simulation(world, seed):
     assert set(owners.tolist()) <= set(range(world))
     computed = sorted(k for _, _, calls, _ in res for (L, g0, g1) in calls for k in range(g0, g1) for _ in [L])
     assert len(computed) == len(t)
+
+
+@pytest.mark.parametrize("world,seed", [(2, 3), (3, 4)])
+def test_level_loop_fused_exchange_matches_simulation(world, seed):
+    """fused exchange: run_level stores every output row into all ranks' arrays (here
+    shared-memory CPU tensors stand in for the CUDA-IPC peer arrays) and the loop takes only a barrier per level;
+    every rank must end with the plaintext simulation's values and identical arrays"""
+    n_in, t, a, b, c = _netlist(seed)
+    import paper_conf_ispass_maxw23_b200 as tb
+    rows_total = tb.Netlist(n_in, t, a, b, c).n_wires
+    shared = [torch.full((rows_total, 3), -1, dtype=torch.int32).share_memory_() for _ in range(world)]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, seed, q, shared)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    bits = np.random.default_rng(seed).integers(0, 2, n_in)
+    want = simulate(n_in, t, a, b, c, bits)[0]
+    for rank, w, calls, rows in res:
+        assert (w[rows, 0] == want).all(), "rank %d wire values differ from the plaintext simulation" % rank
+    for _, w, _, _ in res[1:]:
+        assert (w == res[0][1]).all()
+    assert sum(g1 - g0 for _, _, calls, _ in res for (L, g0, g1) in calls) == len(t)
 
 
 def test_shard_and_slack():

@@ -1,7 +1,8 @@
 """Multi-rank execution of real netlists on the GPU kernels (-m gpu): R = 2 and 3 processes share the one
-B200 of the test box, each running its shard of every level through tb_run_level, with the in-place all-gather
-of the level's output rows done by torch.distributed (gloo on CUDA tensors here; NCCL on a multi-GPU box --
-the level loop, paper_conf_ispass_maxw23_b200.parallel.level_loop, is the same code).  Every rank's wire array
+B200 of the test box, each running its shard of every level through tb_run_level, with the level's output rows
+exchanged either by an in-place all-gather in torch.distributed (gloo on CUDA tensors here; NCCL on a
+multi-GPU box -- the level loop, paper_conf_ispass_maxw23_b200.parallel.level_loop, is the same code) or by the
+fused all-gather (key-switch stores into the other ranks' arrays, mapped with CUDA IPC).  Every rank's wire array
 must equal the oracle's level-by-level evaluation byte for byte (R-invariance).
 """
 import os
@@ -31,7 +32,7 @@ def _netlist():
     return dict(n_inputs=n_in, type=t, in0=a, in1=b, in2=c)
 
 
-def _worker(rank, world, port, keyfile, ctsfile, q):
+def _worker(rank, world, port, keyfile, ctsfile, q, exchange):
     import torch
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -48,15 +49,17 @@ def _worker(rank, world, port, keyfile, ctsfile, q):
         wires = ctx.wire_array(dnet, slack_rows=tb.slack_rows(dnet, world))
         cts = np.load(ctsfile)
         wires[:n["n_inputs"], :631] = ctx.to_device(cts)[:, :631]
-        ctx.run_netlist(dnet, wires, group=dist.group.WORLD)
+        ctx.run_netlist(dnet, wires, group=dist.group.WORLD, exchange=exchange)
         torch.cuda.synchronize()
         q.put((rank, ctx.to_host(wires[:dnet.n_rows])[dnet.row_of_wire]))
     finally:
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world", [2, 3])
-def test_sharded_netlist_matches_oracle(world):
+@pytest.mark.parametrize("world,exchange", [(2, "allgather"), (3, "allgather"), (2, "fused"), (3, "fused")])
+def test_sharded_netlist_matches_oracle(world, exchange):
+    """exchange="fused": the key-switch kernels store each output row into every rank's wire array through CUDA
+    IPC peer mappings (the fused all-gather; same-device IPC between processes here, NVLink peers on a box)"""
     import torch
     import torch.multiprocessing as mp
     if not torch.cuda.is_available():
@@ -73,7 +76,7 @@ def test_sharded_netlist_matches_oracle(world):
         ctx = mp.get_context("spawn")
         q = ctx.Queue()
         port = _port()
-        procs = [ctx.Process(target=_worker, args=(r, world, port, kf, cf, q)) for r in range(world)]
+        procs = [ctx.Process(target=_worker, args=(r, world, port, kf, cf, q, exchange)) for r in range(world)]
         for p in procs:
             p.start()
         res = [q.get(timeout=600) for _ in range(world)]
