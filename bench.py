@@ -163,6 +163,9 @@ def main():
     ap.add_argument("--lanes-per-cta", type=int, default=2)
     ap.add_argument("--br-variant", type=int, default=6, choices=[6, 7, 8, 10])
     ap.add_argument("--ks-tile", type=int, default=8, choices=[8, 16, 32])
+    ap.add_argument("--exchange", default="fused", choices=["fused", "allgather"],
+                    help="N > 1: per-level exchange of output rows (fused into the key switch over NVLink peer "
+                         "memory, or an NCCL all-gather)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -204,8 +207,16 @@ def main():
     gen.manual_seed(14)
     wires[:n["n_inputs"]].random_(-2 ** 31, 2 ** 31 - 1, generator=gen)     # resident inputs (> L2)
 
+    exchange = args.exchange
+    if group is not None and exchange == "fused":
+        try:
+            ctx.attach_peers(wires, group)
+        except Exception as e:                       # no peer access between the GPUs: NCCL all-gather instead
+            print("fused exchange unavailable (%s); using the NCCL all-gather" % e, file=sys.stderr)
+            exchange = "allgather"
+
     def step():
-        ctx.run_netlist(dnet, wires, group)
+        ctx.run_netlist(dnet, wires, group, exchange=exchange)
 
     for _ in range(args.warmup):
         step()
@@ -338,7 +349,10 @@ def main():
             "vs_baseline": None, "dtype": "u32",
             "data": "synthetic: seeded uniform key material and ciphertexts (evaluation is data-oblivious, P:160)",
             "config": {"workload": workload_name(G), "gates_per_gpu": G, "total_gates": total,
-                       "parallelism": "dp%d (level sharded, NCCL all-gather of output rows)" % world,
+                       "parallelism": "dp%d (level sharded; output rows exchanged %s)" % (
+                           world, "by the key-switch kernels' stores into every GPU's wire array (NVLink peer "
+                                  "memory) + NCCL barrier" if exchange == "fused" else "by an NCCL all-gather"),
+                       "exchange": exchange if world > 1 else None,
                        "lanes_per_cta": args.lanes_per_cta, "br_variant": args.br_variant,
                        "l2": "inputs larger than L2 (%.0f MB of input ciphertexts per GPU)" % (2 * G * 2524 / 1e6)},
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,

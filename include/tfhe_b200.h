@@ -133,13 +133,13 @@ int tb_netlist_level(const tb_dev_netlist* dnet, int64_t level, int64_t* row0, i
 int tb_run_level(tb_ctx* ctx, const tb_dev_netlist* dnet, int64_t level, int64_t g0, int64_t g1,
                  uint32_t* wires, int64_t stride, tb_stream stream);
 /* Fused all-gather for the multi-GPU level loop (the paper's per-level exchange of output
- * ciphertexts): after this call, the key-switch kernels of tb_run_level store every output row not only
- * into `wires` but, at the same row offset, into each of the n arrays peer_wires[0..n-1] (HOST array of DEVICE
- * pointers valid in this process: the other ranks' wire arrays, opened with tb_ipc_import; same rows and
- * stride as the `wires` passed to tb_run_level).  The transfer rides on the key switch's own stores (NVLink
+ * ciphertexts): after this call, the key-switch kernels of tb_run_level calls on the DEVICE array
+ * `own_wires` store every output row not only there but, at the same row offset, into each of the n arrays
+ * peer_wires[0..n-1] (HOST array of DEVICE pointers valid in this process: the other ranks' wire arrays,
+ * opened with tb_ipc_import; same rows and stride).  Runs on any other wire array are unaffected.  The transfer rides on the key switch's own stores (NVLink
  * peer writes), so each level needs only a barrier across ranks instead of an all-gather.  n = 0 disables.
  * The caller keeps the peer mappings alive while set.  Errors: TB_EINVAL (n < 0, null pointers), TB_ECUDA. */
-int tb_set_peer_wires(tb_ctx* ctx, uint32_t* const* peer_wires, int n);
+int tb_set_peer_wires(tb_ctx* ctx, const uint32_t* own_wires, uint32_t* const* peer_wires, int n);
 #define TB_IPC_HANDLE_BYTES 64
 /* CUDA IPC export of a device pointer: handle (TB_IPC_HANDLE_BYTES bytes, caller-owned) of the allocation
  * containing dev_ptr and dev_ptr's byte offset in it.  Errors: TB_EINVAL, TB_ECUDA. */

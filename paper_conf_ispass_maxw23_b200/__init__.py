@@ -260,36 +260,50 @@ class Context:
         R, r = dist.get_world_size(group), dist.get_rank(group)
         h = (ctypes.c_ubyte * 64)()
         off = ctypes.c_int64()
-        _native.check(_native.lib().tb_ipc_export(_ptr(wires), h, ctypes.byref(off)))
-        mine = (bytes(h), off.value, tuple(wires.shape), wires.stride(0))
-        allh = [None] * R
-        dist.all_gather_object(allh, mine, group=group)
-        ptrs, bases = [], []
+        mine, err = None, None
         try:
-            for k, (hb, o, shape, stride) in enumerate(allh):
-                if k == r:
-                    continue
-                if shape != tuple(wires.shape) or stride != wires.stride(0):
-                    raise ValueError("rank %d's wire array has shape %s / stride %d, not %s / %d"
-                                     % (k, shape, stride, tuple(wires.shape), wires.stride(0)))
-                p, b = ctypes.c_void_p(), ctypes.c_void_p()
-                buf = (ctypes.c_ubyte * 64).from_buffer_copy(hb)
-                _native.check(_native.lib().tb_ipc_import(self._h, buf, o, ctypes.byref(p), ctypes.byref(b)))
-                ptrs.append(p.value)
-                bases.append(b.value)
-            arr = (ctypes.c_void_p * max(len(ptrs), 1))(*ptrs)
-            _native.check(_native.lib().tb_set_peer_wires(self._h, arr, len(ptrs)))
-        except Exception:
+            _native.check(_native.lib().tb_ipc_export(_ptr(wires), h, ctypes.byref(off)))
+            mine = (bytes(h), off.value, tuple(wires.shape), wires.stride(0))
+        except TBError as e:
+            err = str(e)
+        allh = [None] * R
+        dist.all_gather_object(allh, mine, group=group)     # collective: every rank takes part, even on failure
+        ptrs, bases = [], []
+        err = None if mine is not None else err
+        if err is None and any(x is None for x in allh):
+            err = "a peer rank could not export its wire array"
+        if err is None:
+            try:
+                for k, (hb, o, shape, stride) in enumerate(allh):
+                    if k == r:
+                        continue
+                    if shape != tuple(wires.shape) or stride != wires.stride(0):
+                        raise ValueError("rank %d's wire array has shape %s / stride %d, not %s / %d"
+                                         % (k, shape, stride, tuple(wires.shape), wires.stride(0)))
+                    p, b = ctypes.c_void_p(), ctypes.c_void_p()
+                    buf = (ctypes.c_ubyte * 64).from_buffer_copy(hb)
+                    _native.check(_native.lib().tb_ipc_import(self._h, buf, o, ctypes.byref(p), ctypes.byref(b)))
+                    ptrs.append(p.value)
+                    bases.append(b.value)
+                arr = (ctypes.c_void_p * max(len(ptrs), 1))(*ptrs)
+                _native.check(_native.lib().tb_set_peer_wires(self._h, _ptr(wires), arr, len(ptrs)))
+            except (TBError, ValueError) as e:
+                err = str(e)
+        oks = [None] * R
+        dist.all_gather_object(oks, err is None, group=group)   # all ranks attach, or none does
+        if not all(oks):
+            _native.lib().tb_set_peer_wires(self._h, None, None, 0)
             for b in bases:
                 _native.lib().tb_ipc_close(self._h, ctypes.c_void_p(b))
-            raise
+            raise TBError(_native.TB_ECUDA,
+                          "fused exchange unavailable: %s" % (err or "failed on another rank"))
         self._peer_bases, self._peer_key = bases, key
 
     def detach_peers(self):
         """Stop storing into peer arrays and unmap them."""
         bases = getattr(self, "_peer_bases", [])
         if getattr(self, "_h", None):
-            _native.check(_native.lib().tb_set_peer_wires(self._h, None, 0))
+            _native.check(_native.lib().tb_set_peer_wires(self._h, None, None, 0))
             for b in bases:
                 _native.lib().tb_ipc_close(self._h, ctypes.c_void_p(b))
         self._peer_bases, self._peer_key = [], None

@@ -80,7 +80,7 @@ SIGNATURES = {
     "tb_netlist_level": (ctypes.c_int, [_vp, _i64, _pi64, _pi64, _pi64, _pi64]),
     "tb_run_level": (ctypes.c_int, [_vp, _vp, _i64, _i64, _i64, _vp, _i64, _vp]),
     "tb_run_netlist": (ctypes.c_int, [_vp, _vp, _vp, _i64, _vp]),
-    "tb_set_peer_wires": (ctypes.c_int, [_vp, _vp, ctypes.c_int]),
+    "tb_set_peer_wires": (ctypes.c_int, [_vp, _vp, _vp, ctypes.c_int]),
     "tb_ipc_export": (ctypes.c_int, [_vp, _vp, _pi64]),
     "tb_ipc_import": (ctypes.c_int, [_vp, _vp, _i64, ctypes.POINTER(_vp), ctypes.POINTER(_vp)]),
     "tb_ipc_close": (ctypes.c_int, [_vp, _vp]),

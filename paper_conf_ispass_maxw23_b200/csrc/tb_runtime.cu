@@ -94,6 +94,7 @@ struct tb_ctx {
     int64_t hidx_n = 0;
     uint32_t** peers = nullptr;             // fused all-gather: device array of the other ranks' wire bases
     int32_t npeers = 0;
+    const uint32_t* peer_own = nullptr;     // the local wire array the peers mirror (other arrays: no peer stores)
     uint32_t* ks_scratch = nullptr;         // split key-switch partial sums (narrow levels)
     size_t ks_scratch_words = 0;
     // per-kernel event timing (tb_profile_*)
@@ -869,26 +870,29 @@ extern "C" int tb_run_level(tb_ctx* c, const tb_dev_netlist* d, int64_t level, i
     if ((rc = grow_lanes(c, std::max<int64_t>(l1 - l0, 1)))) return rc;
     cudaStream_t st = (cudaStream_t)stream;
     if ((rc = run_br(c, wires, wires, wires, stride, d->ldesc + l0, l1 - l0, c->lanebuf, kLaneStride, st))) return rc;
+    const bool mirror = c->npeers > 0 && wires == c->peer_own;
     return run_ks(c, c->lanebuf, l0, kLaneStride, d->gdesc + G0, G1 - G0, wires, stride, wires, stride, st,
-                  c->peers, c->npeers);
+                  mirror ? c->peers : nullptr, mirror ? c->npeers : 0);
 }
 
 // ------------------------------------------------------------------------------------------ fused all-gather
 // The multi-GPU level loop's exchange step: instead of a per-level NCCL all-gather, the
 // key-switch kernels store every output row into all ranks' wire arrays over NVLink (peer memory opened with
 // CUDA IPC), so the transfer overlaps the key switch tile by tile; the loop then only needs a barrier.
-extern "C" int tb_set_peer_wires(tb_ctx* c, uint32_t* const* peer_wires, int n) {
-    if (!c || n < 0 || (n > 0 && !peer_wires)) return fail(TB_EINVAL, "bad peer list");
+extern "C" int tb_set_peer_wires(tb_ctx* c, const uint32_t* own_wires, uint32_t* const* peer_wires, int n) {
+    if (!c || n < 0 || (n > 0 && (!peer_wires || !own_wires))) return fail(TB_EINVAL, "bad peer list");
     for (int k = 0; k < n; k++)
         if (!peer_wires[k]) return fail(TB_EINVAL, "null peer wire array");
     TB_CUDA(cudaSetDevice(c->device));
     cudaFree(c->peers);
     c->peers = nullptr;
     c->npeers = 0;
+    c->peer_own = nullptr;
     if (n == 0) return TB_OK;
     TB_CUDA(cudaMalloc(&c->peers, (size_t)n * sizeof(uint32_t*)));
     TB_CUDA(cudaMemcpy(c->peers, peer_wires, (size_t)n * sizeof(uint32_t*), cudaMemcpyHostToDevice));
     c->npeers = n;
+    c->peer_own = own_wires;
     return TB_OK;
 }
 
