@@ -13,6 +13,18 @@ namespace tb {
 
 constexpr int kKsThreads = 160;                  // 158 threads x 4 words = 632 words
 
+// words k0..k0+3 (<= n) of an output row: one 16-byte store when aligned (whole-line NVLink writes for the
+// peer copies), else scalar
+__device__ __forceinline__ void store_row4(uint32_t* d, const uint32_t (&v)[4], int k0) {
+    if (k0 + 3 <= kn && (reinterpret_cast<uintptr_t>(d) & 15) == 0) {
+        *reinterpret_cast<uint4*>(d) = make_uint4(v[0], v[1], v[2], v[3]);
+    } else {
+#pragma unroll
+        for (int q = 0; q < 4; q++)
+            if (k0 + q <= kn) d[q] = v[q];
+    }
+}
+
 template <int T>
 __global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A) {
     extern __shared__ __align__(128) unsigned char ks_smem[];
@@ -86,16 +98,9 @@ __global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A) {
             const int gi = g0 + g;
             if (gi < A.ngates) {
                 const int64_t off = (int64_t)A.gates[gi].out_row * A.out_stride;
-                uint32_t* o = A.out + off;
-#pragma unroll
-                for (int q = 0; q < 4; q++)
-                    if (k0 + q <= kn) o[k0 + q] = acc[g][q];
-                for (int p = 0; p < A.npeers; p++) {   // fused all-gather: the same row into every peer's array
-                    uint32_t* po = A.peers[p] + off;
-#pragma unroll
-                    for (int q = 0; q < 4; q++)
-                        if (k0 + q <= kn) po[k0 + q] = acc[g][q];
-                }
+                store_row4(A.out + off + k0, acc[g], k0);
+                for (int p = 0; p < A.npeers; p++)     // fused all-gather: the same row into every peer's array
+                    store_row4(A.peers[p] + off + k0, acc[g], k0);
             }
         }
         if (A.npeers) __threadfence_system();
