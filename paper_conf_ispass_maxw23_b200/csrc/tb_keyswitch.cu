@@ -112,11 +112,12 @@ __global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A) {
 // groups one after another.  Here CTA (g, s) owns input coefficients i in slice s of [0, N) for gate g and writes
 // its partial sum (words mod 2^32) to scratch; ks_reduce_kernel adds the S partials (integer sums mod 2^32 are
 // order-independent, so the result is bit-identical to the tiled kernel).
-constexpr int kKsSplit = 16;
+constexpr int kKsSplitMin = 16;                  // slices per gate: 16, or 32 / 64 for levels of <= 9 / 4 gates
+__host__ __device__ constexpr int ks_split_count(int64_t ngates) { return ngates <= 4 ? 64 : ngates <= 9 ? 32 : 16; }
 
-__global__ void __launch_bounds__(kKsThreads) ks_split_kernel(KsArgs A, uint32_t* __restrict__ partial) {
-    constexpr int I = kN / kKsSplit;
-    __shared__ uint16_t sW[I];
+__global__ void __launch_bounds__(kKsThreads) ks_split_kernel(KsArgs A, uint32_t* __restrict__ partial, int S) {
+    const int I = kN / S;
+    __shared__ uint16_t sW[kN / kKsSplitMin];
     __shared__ uint32_t sB;
     const int tid = threadIdx.x, gi = blockIdx.x, s = blockIdx.y;
     const GateDesc gd = A.gates[gi];
@@ -165,17 +166,17 @@ __global__ void __launch_bounds__(kKsThreads) ks_split_kernel(KsArgs A, uint32_t
             }
         }
     }
-    *reinterpret_cast<uint4*>(partial + ((size_t)gi * kKsSplit + s) * kKsRow + k0) = make_uint4(acc[0], acc[1], acc[2], acc[3]);
+    *reinterpret_cast<uint4*>(partial + ((size_t)gi * S + s) * kKsRow + k0) = make_uint4(acc[0], acc[1], acc[2], acc[3]);
 }
 
-__global__ void __launch_bounds__(kKsThreads) ks_reduce_kernel(KsArgs A, const uint32_t* __restrict__ partial) {
+__global__ void __launch_bounds__(kKsThreads) ks_reduce_kernel(KsArgs A, const uint32_t* __restrict__ partial, int S) {
     const int gi = blockIdx.x;
     const int64_t off = (int64_t)A.gates[gi].out_row * A.out_stride;
     uint32_t* o = A.out + off;
     for (int k = threadIdx.x; k <= kn; k += kKsThreads) {
         uint32_t v = 0u;
 #pragma unroll
-        for (int s = 0; s < kKsSplit; s++) v += partial[((size_t)gi * kKsSplit + s) * kKsRow + k];
+        for (int s = 0; s < S; s++) v += partial[((size_t)gi * S + s) * kKsRow + k];
         o[k] = v;
         for (int p = 0; p < A.npeers; p++) A.peers[p][off + k] = v;   // fused all-gather
     }
@@ -184,11 +185,12 @@ __global__ void __launch_bounds__(kKsThreads) ks_reduce_kernel(KsArgs A, const u
 
 int launch_ks_split(const KsArgs& A, uint32_t* partial, cudaStream_t st) {
     if (A.ngates <= 0) return 0;
-    ks_split_kernel<<<dim3(A.ngates, kKsSplit), kKsThreads, 0, st>>>(A, partial);
-    ks_reduce_kernel<<<A.ngates, kKsThreads, 0, st>>>(A, partial);
+    const int S = ks_split_count(A.ngates);
+    ks_split_kernel<<<dim3(A.ngates, S), kKsThreads, 0, st>>>(A, partial, S);
+    ks_reduce_kernel<<<A.ngates, kKsThreads, 0, st>>>(A, partial, S);
     return 0;
 }
-size_t ks_split_scratch_words(int64_t ngates) { return (size_t)ngates * kKsSplit * kKsRow; }
+size_t ks_split_scratch_words(int64_t ngates) { return (size_t)ngates * ks_split_count(ngates) * kKsRow; }
 
 // digit-0 rows dropped, rows padded to 632 words: [i][j][d][631] (host layout) -> [i][j][d-1][632]
 __global__ void ksk_relayout_kernel(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst) {

@@ -152,11 +152,12 @@ def test_structured_key_closed_form(tb):
 
 
 # ------------------------------------------------------------------------------------- key switch
-@pytest.mark.parametrize("narrow", [148, 0])
-def test_keyswitch_bit_exact(tb, ctx, keys, narrow):
-    """split key switch (narrow levels, 16 CTAs per gate) and tiled key switch (ragged: 4 tiles of 8 + 5)"""
-    rng = np.random.default_rng(6)
-    ext = rng.integers(0, M32, (37, 1025), dtype=np.uint64).astype(np.uint32)
+@pytest.mark.parametrize("narrow,count", [(148, 37), (0, 37), (148, 3), (148, 7)])
+def test_keyswitch_bit_exact(tb, ctx, keys, narrow, count):
+    """split key switch (narrow levels: 16 CTAs per gate at 37 gates, 64 at 3, 32 at 7) and tiled key switch
+    (ragged: 4 tiles of 8 + 5)"""
+    rng = np.random.default_rng(6 + count)
+    ext = rng.integers(0, M32, (count, 1025), dtype=np.uint64).astype(np.uint32)
     ext[0, :] = 0
     ext[1, :1024] = 0xFFFFFFFF
     dev = ctx.to_device(ext, stride=1028)
