@@ -169,6 +169,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--one-gpu-ranks", action="store_true",
+                    help="functional check of the N > 1 path on a one-GPU box: every rank on cuda:0, gloo process "
+                         "group (the numbers are not a scaling measurement)")
     args = ap.parse_args()
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -187,10 +190,15 @@ def main():
     import synth
 
     tb.build()                                        # no-op when the in-tree .so is current
+    if args.one_gpu_ranks:
+        local = 0
     torch.cuda.set_device(local)
     group = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.one_gpu_ranks:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         group = dist.group.WORLD
     G = args.gates_per_gpu
     total = G * world
