@@ -248,6 +248,45 @@ def test_edge_cases(tb, ctx, keys):
         ctx.gates(tb.NAND, ctx.to_device(one_a))                            # missing cb
 
 
+def test_peer_exchange_api_errors_and_scope(tb, ctx, keys):
+    """fused-exchange plumbing: bad arguments fail loudly (TB_EINVAL), a handle exports, and with a peer array
+    registered a run on another wire array (here tb_run_netlist_host) does not
+    store into the peer (the mirror is scoped to the registered array)"""
+    import ctypes
+    import torch
+    from paper_conf_ispass_maxw23_b200 import _native
+    L = _native.lib()
+    h = (ctypes.c_ubyte * 64)()
+    off = ctypes.c_int64()
+    assert L.tb_ipc_export(None, h, ctypes.byref(off)) == _native.TB_EINVAL
+    assert L.tb_set_peer_wires(ctx._h, None, None, -1) == _native.TB_EINVAL
+    assert L.tb_set_peer_wires(ctx._h, None, None, 1) == _native.TB_EINVAL
+    w = ctx.empty(8)
+    assert L.tb_ipc_export(ctypes.c_void_p(w.data_ptr()), h, ctypes.byref(off)) == 0
+    assert L.tb_ipc_import(ctx._h, None, 0, None, None) == _native.TB_EINVAL
+    # register `mirror` as the "peer" of `own`; a host-buffer run (context-owned wire array) must not touch it
+    n = synth.independent_level(4, 2)
+    net = tb.Netlist(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"], outputs=n["outputs"])
+    dnet = ctx.upload(net)
+    own, mirror = ctx.wire_array(dnet), ctx.wire_array(dnet)
+    mirror.fill_(7)
+    arr = (ctypes.c_void_p * 1)(mirror.data_ptr())
+    assert L.tb_set_peer_wires(ctx._h, ctypes.c_void_p(own.data_ptr()), arr, 1) == 0
+    try:
+        cts = enc(keys, synth.random_bits(n["n_inputs"], 3), 4)
+        ctx.run_netlist_host(dnet, cts, n["outputs"])
+        torch.cuda.synchronize()
+        assert bool((mirror == 7).all())
+        own[:n["n_inputs"], :631] = ctx.to_device(cts)[:, :631]
+        ctx.run_netlist(dnet, own)                  # the registered array: every output row mirrored
+        torch.cuda.synchronize()
+        rows = slice(n["n_inputs"], dnet.n_rows)
+        assert bool((mirror[rows, :631] == own[rows, :631]).all())
+    finally:
+        assert L.tb_set_peer_wires(ctx._h, None, None, 0) == 0
+    dnet.free()
+
+
 def test_host_buffer_path_matches(tb, ctx, keys):
     A, B = synth.random_bits(9, 90), synth.random_bits(9, 91)
     ca, cb = enc(keys, A, 92), enc(keys, B, 93)
