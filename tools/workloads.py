@@ -69,7 +69,8 @@ def main():
                           "level_ms_median": round(float(np.median(best)), 3),
                           "level_ms_p90": round(float(np.percentile(best, 90)), 3),
                           "level_ms_max": round(float(best.max()), 3),
-                          "gates_per_s": round(d.n_boot / tot * 1e3, 1)}), flush=True)
+                          "gates_per_s": round(d.n_boot / tot * 1e3, 1),
+                          "bootstraps_per_s": round(sum(lv[3] for lv in d.levels) / tot * 1e3, 1)}), flush=True)
         d.free()
         del w
         torch.cuda.empty_cache()
