@@ -1,6 +1,8 @@
 #!/usr/bin/env python
-"""Small run of every kernel (all blind-rotation variants, latency mode, key switch, a mixed netlist) for
+"""Small run of every kernel (all blind-rotation variants, every latency-mode kernel, tiled and split key
+switch at 3 / 7 / 37 gates, a mixed netlist, and the fused-exchange peer stores into a second array) for
 compute-sanitizer:  compute-sanitizer --tool {memcheck,racecheck,synccheck} python tools/sanitize_run.py"""
+import ctypes
 import os
 import sys
 
@@ -18,21 +20,37 @@ g.manual_seed(3)
 ct = ctx.empty(5)
 ct.random_(-2 ** 31, 2 ** 31 - 1, generator=g)
 outs = []
-for variant in (6, 7, 8):
+QUICK = os.environ.get("TB_SAN_QUICK") == "1"                # racecheck: key switch, netlist and peer stores only
+for variant in ((6,) if QUICK else (6, 7, 8, 10)):
     ctx.set_br_variant(variant)
     ctx.set_narrow_lanes(0)
     outs.append(ctx.bootstrap_wo_ks(ct))
 ctx.set_br_variant(6)
 ctx.set_narrow_lanes(148)
-outs.append(ctx.bootstrap_wo_ks(ct))                        # latency mode (br7<1>)
-ks = ctx.keyswitch(outs[0])
+for k in (() if QUICK else (11, 9, 7)):                      # latency mode: brl, br9, br7<1>
+    ctx.set_narrow_kernel(k)
+    outs.append(ctx.bootstrap_wo_ks(ct))
+ctx.set_narrow_kernel(0)
+ext = ctx.empty(37, stride=1028)
+ext.random_(-2 ** 31, 2 ** 31 - 1, generator=g)
+ks = [ctx.keyswitch(ext[:c]) for c in (3, 7, 37)]           # split KS: 64 / 32 / 16 slices per gate
+ctx.set_narrow_lanes(0)
+ks.append(ctx.keyswitch(ext))                               # tiled KS
+ctx.set_narrow_lanes(148)
 n = synth.ripple_carry_adder(2)
 net = tb.Netlist(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"])
 d = ctx.upload(net)
 w = ctx.wire_array(d)
 w[:n["n_inputs"]].random_(-2 ** 31, 2 ** 31 - 1, generator=g)
 ctx.run_netlist(d, w)
+mirror = ctx.wire_array(d)                                  # fused exchange: peer stores into a second array
+arr = (ctypes.c_void_p * 1)(mirror.data_ptr())
+tb._native.check(tb._native.lib().tb_set_peer_wires(ctx._h, ctypes.c_void_p(w.data_ptr()), arr, 1))
+ctx.run_netlist(d, w)
+tb._native.check(tb._native.lib().tb_set_peer_wires(ctx._h, None, None, 0))
 torch.cuda.synchronize()
+same_rows = torch.equal(mirror[n["n_inputs"]:d.n_rows, :631], w[n["n_inputs"]:d.n_rows, :631])
+print("peer mirror equal:", same_rows)
 same = all(torch.equal(outs[0][:, :1025], o[:, :1025]) for o in outs[1:])
 print("variants agree:", same)
-sys.exit(0 if same else 1)
+sys.exit(0 if same and same_rows else 1)
