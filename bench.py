@@ -216,6 +216,7 @@ def main():
     wires[:n["n_inputs"]].random_(-2 ** 31, 2 ** 31 - 1, generator=gen)     # resident inputs (> L2)
 
     exchange = args.exchange
+    coll = "gloo (--one-gpu-ranks functional check)" if args.one_gpu_ranks else "NCCL"
     if group is not None and exchange == "fused":
         try:
             ctx.attach_peers(wires, group)
@@ -359,7 +360,7 @@ def main():
             "config": {"workload": workload_name(G), "gates_per_gpu": G, "total_gates": total,
                        "parallelism": "dp%d (level sharded; output rows exchanged %s)" % (
                            world, "by the key-switch kernels' stores into every GPU's wire array (NVLink peer "
-                                  "memory) + NCCL barrier" if exchange == "fused" else "by an NCCL all-gather"),
+                                  "memory) + %s barrier" % coll if exchange == "fused" else "by a %s all-gather" % coll),
                        "exchange": exchange if world > 1 else None,
                        "lanes_per_cta": args.lanes_per_cta, "br_variant": args.br_variant,
                        "l2": "inputs larger than L2 (%.0f MB of input ciphertexts per GPU)" % (2 * G * 2524 / 1e6)},
