@@ -20,7 +20,8 @@
 
 namespace tb {
 
-constexpr int kLThreads = 192;                 // 6 warps: 3 forward transforms x 2 warps; warps 0-1 invert
+constexpr int kLThreads = 256;                 // 8 warps: 3 forward transforms x 2 warps (0-5); warps 0-1 invert; all MAC
+constexpr int kLMacIt = (512 + kLThreads - 1) / kLThreads;
 
 #ifdef TB_BRL_TRACE   // scratch instrumentation (tools/buildvar.sh WORK name -DTB_BRL_TRACE): clock64 per phase
 __device__ long long g_brl_trace[4][8][16];
@@ -234,7 +235,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
 
     const int tt = (warp & 1) * 32 + lane;               // thread index within its warp pair
     const int jd = warp >> 1;                             // forward role: digit jd of bloc q (warps 0-5)
-    const int shift = 32 - kBgbit * (jd + 1);
+    const int shift = 32 - kBgbit * (jd < kL ? jd + 1 : 1);
     PassTw t1, t2, t3;
     t1.a = dcplx{c_zeta[0].x, c_zeta[0].y};
     t1.b = dcplx{c_zeta[1].x, c_zeta[1].y};
@@ -254,7 +255,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         const int buf = i & 1;
         const uint32_t par = (uint32_t)((i >> 1) & 1);
         BRL_T(0)
-        {   // ---- A: digit jd of (X^abar - 1) ACC[q], folded, forward transform (warp pair jd) ----
+        if (jd < kL) {   // ---- A: digit jd of (X^abar - 1) ACC[q], folded, forward transform (warp pair jd) ----
             const uint32_t ab = S.bar[i];
             const uint32_t* win = S.acc + ((tt - (int)ab) & (kTwoN - 1));
             dcplx x[8];
@@ -276,9 +277,9 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         mb_wait(&S.mbar_bk[buf], par);
         BRL_T(2)
         // ---- B: out[k] = sum_{r<6} D_r[k] BK_i[r][o][k]; own bloc's rows first, then the other bloc's ----
-        dcplx m3[3];
+        dcplx m3[kLMacIt];
 #pragma unroll
-        for (int e = 0; e < 3; e++) {
+        for (int e = 0; e < kLMacIt; e++) {
             const int k = tid + kLThreads * e;
             dcplx s = {0.0, 0.0};
             if (k < 512) {
@@ -294,7 +295,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         mb_wait(&S.mbar_rows[buf], par);
         BRL_T(3)
 #pragma unroll
-        for (int e = 0; e < 3; e++) {
+        for (int e = 0; e < kLMacIt; e++) {
             const int k = tid + kLThreads * e;
             if (k < 512) {
                 dcplx s = m3[e];
