@@ -341,11 +341,11 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         }
         __syncthreads();                                  // rres[buf] consumed
         BRL_T(7)
-        if (tid == 0) {
+        if (tid == 0) {   // (no barrier after this: warps 0-1 rewrite res only after the next phase-A barrier,
+                          // which tid 0 reaches after the wait; the expect precedes tid 0's own next push)
             asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // res readable again
             if (i + 2 < kn) mb_expect(&S.mbar_res[buf], kN * 4);            // the sibling's half of step i + 2
         }
-        __syncthreads();
     }
     cl_sync();
     if (gl < A.nlanes && h == 0) {   // a5: CTA (0, 0) holds ACC.a, CTA (1, 0) holds ACC.b
