@@ -21,6 +21,7 @@ namespace tb {
 
 constexpr int kB9HalfWords = kRows * kParts * kN;          // 18,432 words = 72 KB per CTA per step
 constexpr int kB9RowWords = kL * 32 * 32;                   // 3 rows = 12 KB
+constexpr int kB9Threads = 256;                             // 8 warps: 0-2 transform, all 8 MAC (4 coefficients each)
 
 struct __align__(128) Br9Smem {
     uint32_t bk[2][kB9HalfWords];       // [step & 1][r][m][a] for this CTA's output q = c
@@ -77,7 +78,7 @@ __device__ __forceinline__ void issue_bk9(Br9Smem& S, const uint32_t* bkhat, int
             : "memory");
 }
 
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1) br9_kernel(BrArgs A) {
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kB9Threads, 1) br9_kernel(BrArgs A) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     Br9Smem& S = *reinterpret_cast<Br9Smem*>(smem_raw);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -98,7 +99,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1) br9_kernel(B
         issue_bk9(S, A.bkhat, 0, (int)c, 0);
         issue_bk9(S, A.bkhat, 1, (int)c, 1);
     }
-    for (int k = tid; k < 31 * 32; k += 192) {
+    for (int k = tid; k < 31 * 32; k += kB9Threads) {
         S.twF[k] = A.twF[k];
         S.twI[k] = A.twI[k];
     }
@@ -110,7 +111,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1) br9_kernel(B
         const uint32_t* s1 = sb == 0 ? A.src0 : (sb == 1 ? A.src1 : A.src2);
         const uint32_t* pa = s0 + (int64_t)d.ia * A.src_stride;
         const uint32_t* pb = d.ib >= 0 ? s1 + (int64_t)d.ib * A.src_stride : nullptr;
-        for (int w = tid; w <= kn; w += 192) {
+        for (int w = tid; w <= kn; w += kB9Threads) {
             uint32_t v = (gl < A.nlanes) ? (uint32_t)d.wa * __ldg(pa + w) : 0u;
             if (pb) v += (uint32_t)d.wb * __ldg(pb + w);
             if (w == kn) v += d.cst;
@@ -118,7 +119,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1) br9_kernel(B
         }
     }
     __syncthreads();
-    for (int k = tid; k < kN; k += 192) {                  // a3: ACC[0] = 0, ACC[1] = X^{-bbar} (mu, ..., mu)
+    for (int k = tid; k < kN; k += kB9Threads) {                  // a3: ACC[0] = 0, ACC[1] = X^{-bbar} (mu, ..., mu)
         const uint32_t bbar = S.bar[kn];
         S.acc[k] = c == 0 ? 0u : (((k + bbar) & (kTwoN - 1)) < (uint32_t)kN ? kMu : (uint32_t)(0u - kMu));
     }
@@ -160,12 +161,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1) br9_kernel(B
         }
         mbar_wait9(&S.mbar_bk[buf], (uint32_t)((i >> 1) & 1));             // BK_i has landed
         // ---- B: out[m][a] = sum_{r<6} D_r[a] BK_i[r][3c + m][a]; own rows first, then the peer's ----
-        constexpr int KMAX = (kN + 191) / 192;
+        constexpr int KMAX = (kN + kB9Threads - 1) / kB9Threads;
         uint64_t acc[KMAX][kParts];
         const uint32_t* bk = S.bk[buf];
 #pragma unroll
         for (int k = 0; k < KMAX; k++) {
-            const int a = tid + 192 * k;
+            const int a = tid + kB9Threads * k;
 #pragma unroll
             for (int m = 0; m < kParts; m++) acc[k][m] = 0ull;
             if (a < kN) {
@@ -182,7 +183,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1) br9_kernel(B
         mbar_wait9(&S.mbar_rows[buf], (uint32_t)((i >> 1) & 1));           // the peer's rows have landed
 #pragma unroll
         for (int k = 0; k < KMAX; k++) {
-            const int a = tid + 192 * k;
+            const int a = tid + kB9Threads * k;
             if (a < kN) {
                 const int sa = sidx<true>(a >> 5, a & 31);
 #pragma unroll
@@ -233,7 +234,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1) br9_kernel(B
     if (gl < A.nlanes) {   // a5: CTA 0 holds ACC.a, CTA 1 holds ACC.b
         uint32_t* o = A.out + (int64_t)gl * A.out_stride;
         if (c == 0) {
-            for (int j = tid; j < kN; j += 192) o[j] = j == 0 ? S.acc[0] : 0u - S.acc[kN - j];
+            for (int j = tid; j < kN; j += kB9Threads) o[j] = j == 0 ? S.acc[0] : 0u - S.acc[kN - j];
         } else if (tid == 0) {
             o[kN] = S.acc[0];
         }
@@ -249,7 +250,7 @@ int launch_br9(const BrArgs& A, cudaStream_t st) {
         attr = true;
     }
     if (A.nlanes <= 0) return 0;
-    br9_kernel<<<2 * A.nlanes, 192, smem, st>>>(A);
+    br9_kernel<<<2 * A.nlanes, kB9Threads, smem, st>>>(A);
     return 0;
 }
 
