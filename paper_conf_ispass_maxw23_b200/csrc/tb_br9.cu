@@ -6,7 +6,7 @@
 //   A  warps 0-2: digit jd of (X^abar - 1) ACC[c] -> forward NTT -> local rows (global rows r = 3c + jd); one
 //      thread pushes the 3 rows (12 KB) into the peer's receive buffer with a shared::cta -> shared::cluster
 //      bulk copy that completes on the peer's mbarrier (double-buffered by step parity)
-//   B  all 6 warps: for output polynomial q = c (3 BK parts): MAC over the 3 local rows, wait for the peer's
+//   B  all 8 warps: for output polynomial q = c (3 BK parts): MAC over the 3 local rows, wait for the peer's
 //      rows, MAC over them (both from local shared memory), reduce
 //   C  warps 0-2: inverse NTT of part m, lift, << 11m; named barrier; warp 0 adds the parts into ACC[c]
 // The output of step i on CTA c is ACC[c] of step i+1, so accumulators never cross the cluster.  Each CTA
