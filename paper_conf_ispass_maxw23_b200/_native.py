@@ -112,7 +112,7 @@ def lib():
     """Load the in-tree shared library (raises if it has not been built)."""
     global _lib
     if _lib is None:
-        path = os.environ.get("TB_LIB", SO_PATH)     # A/B timing of alternative builds (scratch/ab.sh)
+        path = os.environ.get("TB_LIB", SO_PATH)     # A/B timing of alternative builds (tools/ab.sh)
         if not os.path.exists(path):
             raise RuntimeError("%s is not built (run __graft_entry__.build()); there is no CPU fallback" % path)
         L = ctypes.CDLL(path)

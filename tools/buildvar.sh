@@ -1,4 +1,4 @@
-# usage: scratch/buildvar.sh <git-rev|WORK> <name>: build libtfhe_b200.so of that source state into scratch/lib_<name>.so
+# usage: tools/buildvar.sh <git-rev|WORK> <name>: build libtfhe_b200.so of that source state into scratch/lib_<name>.so
 set -e
 D=/tmp/bv_$2; rm -rf $D; mkdir -p $D/pkg
 if [ "$1" = WORK ]; then cp -r /root/repo/paper_conf_ispass_maxw23_b200/csrc $D/pkg/; cp -r /root/repo/include $D/; else
