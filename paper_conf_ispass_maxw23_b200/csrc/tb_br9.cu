@@ -8,7 +8,7 @@
 //      bulk copy that completes on the peer's mbarrier (double-buffered by step parity)
 //   B  all 8 warps: for output polynomial q = c (3 BK parts): MAC over the 3 local rows, wait for the peer's
 //      rows, MAC over them (both from local shared memory), reduce
-//   C  warps 0-2: inverse NTT of part m, lift, << 11m; named barrier; warp 0 adds the parts into ACC[c]
+//   C  warps 0-2: inverse NTT of part m, lift, << 11m; CTA barrier; all 8 warps add the parts into ACC[c]
 // The output of step i on CTA c is ACC[c] of step i+1, so accumulators never cross the cluster.  Each CTA
 // stages the half of BK_i it needs (72 KB) by cp.async.bulk two steps ahead (double buffer).  There is no
 // cluster-wide barrier inside the loop: the two CTAs are coupled only by the row hand-over, which also makes
@@ -215,17 +215,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kB9Threads, 1) br9_k
             for (int j = 0; j < 32; j++) x[j] = slot[sidx<true>(lane, j)];
             ntt_inv<true>(x, slot, S.twI, lane);
 #pragma unroll
-            for (int j = 0; j < 32; j++) x[j] = lift_centred(x[j]) << (11 * m);
-            if (m != 0) {
-#pragma unroll
-                for (int j = 0; j < 32; j++) slot[sidx<true>(j, lane)] = x[j];
-            }
-            asm volatile("bar.sync 1, 96;" ::: "memory");
-            if (m == 0) {
-#pragma unroll
-                for (int j = 0; j < 32; j++)
-                    S.acc[lane + 32 * j] += x[j] + S.oslot[1][sidx<true>(j, lane)] + S.oslot[2][sidx<true>(j, lane)];
-            }
+            for (int j = 0; j < 32; j++) slot[sidx<true>(j, lane)] = lift_centred(x[j]) << (11 * m);
+        }
+        __syncthreads();
+        for (int k = tid; k < kN; k += kB9Threads) {       // ACC[c] += the three parts, over all 8 warps
+            const int sk = sidx<true>(k >> 5, k & 31);
+            S.acc[k] += S.oslot[0][sk] + S.oslot[1][sk] + S.oslot[2][sk];
         }
         if (tid == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // dslot free again
         __syncthreads();
