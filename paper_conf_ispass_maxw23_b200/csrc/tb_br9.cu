@@ -133,18 +133,19 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kB9Threads, 1) br9_k
 
     for (int i = 0; i < kn; i++) {
         const int buf = i & 1;
-        if (warp < kL) {   // ---- A ----
+        {   // ---- A0: (X^abar - 1) ACC[c] + decomposition offset, all 8 warps, into oslot[0] (free until the MAC)
             const uint32_t ab = S.bar[i];
+            for (int k = tid; k < kN; k += kB9Threads) {
+                const uint32_t mm = ((uint32_t)k - ab) & (kTwoN - 1);
+                const uint32_t src = S.acc[mm & (kN - 1)];
+                S.oslot[0][k] = (mm < (uint32_t)kN ? src : 0u - src) - S.acc[k] + kDecompOffset;
+            }
+        }
+        __syncthreads();
+        if (warp < kL) {   // ---- A ----
             uint32_t x[32];
 #pragma unroll
-            for (int j = 0; j < 32; j++) {
-                const uint32_t cc = lane + 32 * j;
-                const uint32_t mm = (cc - ab) & (kTwoN - 1);
-                const uint32_t src = S.acc[mm & (kN - 1)];
-                const uint32_t rot = mm < (uint32_t)kN ? src : 0u - src;
-                const uint32_t u = rot - S.acc[cc] + kDecompOffset;
-                x[j] = ((u >> shift) & 127u) + (kP - 64u);
-            }
+            for (int j = 0; j < 32; j++) x[j] = ((S.oslot[0][lane + 32 * j] >> shift) & 127u) + (kP - 64u);
             ntt_fwd<true>(x, S.dslot[jd], S.twF, lane);
 #pragma unroll
             for (int j = 0; j < 32; j++) S.dslot[jd][sidx<true>(lane, j)] = red_2p(x[j]);
