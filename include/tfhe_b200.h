@@ -195,7 +195,7 @@ int tb_set_narrow_lanes(tb_ctx* ctx, int64_t lanes);
  * else br9), 11 = brl_kernel (one bootstrap per cluster of 4 SMs on the FP64 path: each SM owns one output
  * polynomial and one 16-bit BK half, transforms split over warp pairs; 1.9 ms per level on B200),
  * 9 = br9_kernel (one bootstrap per cluster of 2 SMs, each SM owning one accumulator polynomial, forward-NTT
- * rows exchanged through distributed shared memory; 3.4 ms), 7 = br7<1> (one bootstrap per SM).  All are
+ * rows exchanged through distributed shared memory; 2.8 ms, 74 per wave), 7 = br7<1> (one bootstrap per SM).  All are
  * bit-identical.  Anything else: TB_EINVAL. */
 int tb_set_narrow_kernel(tb_ctx* ctx, int kernel);
 /* Level schedule used by tb_netlist_upload: Algorithm 1 gives every gate its earliest level;
