@@ -21,6 +21,17 @@ ct = ctx.empty(5)
 ct.random_(-2 ** 31, 2 ** 31 - 1, generator=g)
 outs = []
 QUICK = os.environ.get("TB_SAN_QUICK") == "1"                # racecheck: key switch, netlist and peer stores only
+LAT = os.environ.get("TB_SAN_LATENCY") == "1"                # racecheck: the latency kernels on one lane only
+if LAT:
+    one = ct[:1]
+    res = []
+    for k in (11, 9):
+        ctx.set_narrow_kernel(k)
+        res.append(ctx.bootstrap_wo_ks(one))
+    torch.cuda.synchronize()
+    ok = torch.equal(res[0][:, :1025], res[1][:, :1025])
+    print("latency kernels agree:", ok)
+    sys.exit(0 if ok else 1)
 for variant in ((6,) if QUICK else (6, 7, 8, 10)):
     ctx.set_br_variant(variant)
     ctx.set_narrow_lanes(0)
