@@ -47,7 +47,8 @@ void launch_bk_to_ntt(const uint32_t* bk, uint32_t* bkhat, const uint2* twF, uin
                       cudaStream_t st);
 void launch_build_gate_desc(int kind, int32_t wa, int32_t wb, uint32_t cst, int64_t count, LaneDesc* lanes,
                             GateDesc* gates, cudaStream_t st);
-int launch_ks(const KsArgs& A, int tile, cudaStream_t st);
+int launch_ks(const KsArgs& A, int tile, uint32_t* partial, int S, cudaStream_t st);   // S > 1: sliced + reduce
+int ks_tile_slices(int64_t ngates, int tile);
 int launch_ks_split(const KsArgs& A, uint32_t* partial, cudaStream_t st);   // narrow levels
 size_t ks_split_scratch_words(int64_t ngates);
 void launch_ksk_relayout(const uint32_t* src, uint32_t* dst, cudaStream_t st);

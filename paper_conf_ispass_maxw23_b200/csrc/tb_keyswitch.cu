@@ -25,9 +25,12 @@ __device__ __forceinline__ void store_row4(uint32_t* d, const uint32_t (&v)[4], 
     }
 }
 
+// partial != nullptr: CTA (tile, s) covers input coefficients i in slice s of S (blockIdx.y) and writes its
+// partial sums to partial[gate][s][kKsRow] for ks_reduce_kernel (mid-size levels: more CTAs than tiles)
 template <int T>
-__global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A) {
+__global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A, uint32_t* __restrict__ partial, int S) {
     extern __shared__ __align__(128) unsigned char ks_smem[];
+    const int s = blockIdx.y, I = kN / S, i0 = s * I;
     uint16_t (*sW)[T] = reinterpret_cast<uint16_t (*)[T]>(ks_smem);   // [kN][T]: (a_i + 2^15) >> 16 = 8 digits
     uint32_t* sB = reinterpret_cast<uint32_t*>(ks_smem + (size_t)kN * T * 2);
     const int tid = threadIdx.x;
@@ -66,11 +69,11 @@ __global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A) {
             const int k = k0 + q;
             uint32_t v = (k == kn) ? sB[g] : 0u;
             if (isnot && active && k <= kn) v = 0u - __ldg(A.not_src + (int64_t)A.gates[gi].lane0 * A.not_stride + k);
-            acc[g][q] = v;
+            acc[g][q] = s == 0 ? v : 0u;
         }
     }
     if (active) {
-        for (int i = 0; i < kN; i++) {
+        for (int i = i0; i < i0 + I; i++) {
             uint16_t w[T];
 #pragma unroll
             for (int g = 0; g < T; g += 8) {
@@ -96,7 +99,10 @@ __global__ void __launch_bounds__(kKsThreads) ks_kernel(KsArgs A) {
 #pragma unroll
         for (int g = 0; g < T; g++) {
             const int gi = g0 + g;
-            if (gi < A.ngates) {
+            if (gi < A.ngates && partial) {
+                *reinterpret_cast<uint4*>(partial + ((size_t)gi * S + s) * kKsRow + k0) =
+                    make_uint4(acc[g][0], acc[g][1], acc[g][2], acc[g][3]);
+            } else if (gi < A.ngates) {
                 const int64_t off = (int64_t)A.gates[gi].out_row * A.out_stride;
                 store_row4(A.out + off + k0, acc[g], k0);
                 for (int p = 0; p < A.npeers; p++)     // fused all-gather: the same row into every peer's array
@@ -202,7 +208,7 @@ __global__ void ksk_relayout_kernel(const uint32_t* __restrict__ src, uint32_t* 
 }
 
 template <int T>
-static int launch_ks_t(const KsArgs& A, cudaStream_t st) {
+static int launch_ks_t(const KsArgs& A, uint32_t* partial, int S, cudaStream_t st) {
     const size_t smem = (size_t)kN * T * 2 + T * 4;
     static bool attr = false;
     if (!attr) {
@@ -211,16 +217,25 @@ static int launch_ks_t(const KsArgs& A, cudaStream_t st) {
         attr = true;
     }
     const int blocks = (A.ngates + T - 1) / T;
-    ks_kernel<T><<<blocks, kKsThreads, smem, st>>>(A);
+    ks_kernel<T><<<dim3(blocks, S), kKsThreads, smem, st>>>(A, S > 1 ? partial : nullptr, S);
+    if (S > 1) ks_reduce_kernel<<<A.ngates, kKsThreads, 0, st>>>(A, partial, S);
     return 0;
 }
 
-int launch_ks(const KsArgs& A, int tile, cudaStream_t st) {
+// slices per tile so that a mid-size level still fills the GPU: ~4 CTAs per SM (592 on B200) at least
+int ks_tile_slices(int64_t ngates, int tile) {
+    const int64_t tiles = (ngates + tile - 1) / tile;
+    int S = 1;
+    while (S < 16 && tiles * S < 592) S *= 2;
+    return S;
+}
+
+int launch_ks(const KsArgs& A, int tile, uint32_t* partial, int S, cudaStream_t st) {
     if (A.ngates <= 0) return 0;
     switch (tile) {
-        case 8: return launch_ks_t<8>(A, st);
-        case 16: return launch_ks_t<16>(A, st);
-        case 32: return launch_ks_t<32>(A, st);
+        case 8: return launch_ks_t<8>(A, partial, S, st);
+        case 16: return launch_ks_t<16>(A, partial, S, st);
+        case 32: return launch_ks_t<32>(A, partial, S, st);
         default: return -2;
     }
 }

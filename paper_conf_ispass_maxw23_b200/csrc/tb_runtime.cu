@@ -447,19 +447,22 @@ static int run_ks(tb_ctx* c, const uint32_t* lanes, int64_t lane_base, int64_t l
     A.peers = peers;
     A.npeers = npeers;
     const bool split = c->narrow_lanes > 0 && ngates <= c->narrow_lanes;   // narrow level: split each gate's KS
-    if (split && c->ks_scratch_words < ks_split_scratch_words(ngates)) {
+    // mid-size level: tiles sliced over the input coefficients so that the launch still fills the GPU
+    const int slices = split ? 1 : ks_tile_slices(ngates, c->ks_tile);
+    const size_t need = split ? ks_split_scratch_words(std::max<int64_t>(ngates, c->narrow_lanes))
+                              : (slices > 1 ? (size_t)ngates * slices * kKsRow : 0);
+    if (need > c->ks_scratch_words) {
         cudaFree(c->ks_scratch);
         c->ks_scratch = nullptr;
         c->ks_scratch_words = 0;
-        const size_t words = ks_split_scratch_words(std::max<int64_t>(ngates, c->narrow_lanes));
-        if (cudaMalloc(&c->ks_scratch, words * 4) != cudaSuccess) {
+        if (cudaMalloc(&c->ks_scratch, need * 4) != cudaSuccess) {
             cudaGetLastError();
             return fail(TB_ENOMEM, "key-switch scratch allocation failed");
         }
-        c->ks_scratch_words = words;
+        c->ks_scratch_words = need;
     }
     const long slot = prof_begin(c, 1, st);
-    const int rc = split ? launch_ks_split(A, c->ks_scratch, st) : launch_ks(A, c->ks_tile, st);
+    const int rc = split ? launch_ks_split(A, c->ks_scratch, st) : launch_ks(A, c->ks_tile, c->ks_scratch, slices, st);
     prof_end(c, slot, st);
     if (rc) return fail(TB_ECUDA, "key-switch kernel attribute/launch failed");
     cudaError_t e = cudaGetLastError();

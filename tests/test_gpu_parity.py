@@ -152,10 +152,11 @@ def test_structured_key_closed_form(tb):
 
 
 # ------------------------------------------------------------------------------------- key switch
-@pytest.mark.parametrize("narrow,count", [(148, 37), (0, 37), (148, 3), (148, 7)])
+@pytest.mark.parametrize("narrow,count", [(148, 37), (0, 37), (148, 3), (148, 7), (0, 600)])
 def test_keyswitch_bit_exact(tb, ctx, keys, narrow, count):
     """split key switch (narrow levels: 16 CTAs per gate at 37 gates, 64 at 3, 32 at 7) and tiled key switch
-    (ragged: 4 tiles of 8 + 5)"""
+    (ragged: 4 tiles of 8 + 5, each sliced 16 ways over the input coefficients; 600 gates = 75 tiles x 8
+    slices + reduction)"""
     rng = np.random.default_rng(6 + count)
     ext = rng.integers(0, M32, (count, 1025), dtype=np.uint64).astype(np.uint32)
     ext[0, :] = 0
