@@ -160,7 +160,7 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--gates-per-gpu", type=int, default=65536)
-    ap.add_argument("--lanes-per-cta", type=int, default=2)
+    ap.add_argument("--lanes-per-cta", type=int, default=0, help="0 = auto per launch size")
     ap.add_argument("--br-variant", type=int, default=6, choices=[6, 7, 8, 10])
     ap.add_argument("--ks-tile", type=int, default=8, choices=[8, 16, 32])
     ap.add_argument("--exchange", default="fused", choices=["fused", "allgather"],
@@ -204,6 +204,7 @@ def main():
     total = G * world
     ctx = tb.Context(local)
     ctx.set_lanes_per_cta(args.lanes_per_cta)
+    lpc = ctx.br6_lanes_per_cta(G)   # NAND/XOR level: one lane per gate
     ctx.set_br_variant(args.br_variant)
     ctx.set_ks_tile(args.ks_tile)
     ctx.load_keys(synth.random_words(tb.BK_WORDS, 11), synth.random_words(tb.KSK_WORDS, 12))
@@ -285,7 +286,7 @@ def main():
     if os.path.exists(prof_path):
         try:
             pj = json.load(open(prof_path))
-            if (pj.get("lanes") == lanes_per_launch and pj.get("lanes_per_cta") == args.lanes_per_cta
+            if (pj.get("lanes") == lanes_per_launch and pj.get("lanes_per_cta") == lpc
                     and pj.get("br_variant", 6) == args.br_variant):
                 traffic = pj.get("dram_bytes_per_launch")
         except Exception:
@@ -362,7 +363,7 @@ def main():
                            world, "by the key-switch kernels' stores into every GPU's wire array (NVLink peer "
                                   "memory) + %s barrier" % coll if exchange == "fused" else "by a %s all-gather" % coll),
                        "exchange": exchange if world > 1 else None,
-                       "lanes_per_cta": args.lanes_per_cta, "br_variant": args.br_variant,
+                       "lanes_per_cta": lpc, "br_variant": args.br_variant,
                        "l2": "inputs larger than L2 (%.0f MB of input ciphertexts per GPU)" % (2 * G * 2524 / 1e6)},
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
             "gpu_launches": br_n + ks_n,

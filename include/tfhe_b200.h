@@ -181,8 +181,11 @@ int tb_ntt_muladd6(tb_ctx* ctx, const int32_t* digits, const uint32_t* polys, ui
  * halves, rounding to the nearest integer).  Synchronous. */
 int tb_fft_muladd6(tb_ctx* ctx, const int32_t* digits, const uint32_t* polys, uint32_t* res);
 
-/* Blind-rotation lanes per CTA for the default kernel (1..4, default 2); tuning knob. */
+/* Blind-rotation lanes per CTA for the default kernel: 1..4 fixed, or 0 (default) = auto per launch: 1 or 2,
+ * whichever leaves the busiest SM the least work for that lane count. */
 int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
+/* The lanes per CTA the default kernel uses for a launch of `nlanes` lanes (>= 1), or < 0 (TB_EINVAL). */
+int tb_br6_lanes_per_cta(tb_ctx* ctx, int64_t nlanes);
 /* Blind-rotation kernel: 6 = br6_kernel (default: 6 warps/lane, 2 CTAs/SM, BK words from L2), 8 = br8_kernel
  * (two ping-ponged lane groups per CTA), 10 = brf_kernel (FP64-pipe FFT), 7 = br7_kernel
  * (2 lanes/CTA, 1 CTA/SM, each 144 KB BK step TMA-bulk-copied into shared memory one step ahead).  Both are

@@ -116,7 +116,15 @@ class Context:
         self.load_ksk(ksk)
 
     def set_lanes_per_cta(self, lanes: int):
+        """1..4 fixed, 0 = auto per launch (the default)."""
         _native.check(_native.lib().tb_set_lanes_per_cta(self._h, lanes))
+
+    def br6_lanes_per_cta(self, nlanes: int) -> int:
+        """Lanes per CTA the default blind-rotation kernel uses for a launch of `nlanes` lanes."""
+        rc = _native.lib().tb_br6_lanes_per_cta(self._h, nlanes)
+        if rc < 0:
+            _native.check(rc)
+        return rc
 
     def set_br_variant(self, variant: int):
         """6 = br6_kernel (default), 7 = br7_kernel (TMA-staged BK); bit-identical outputs."""

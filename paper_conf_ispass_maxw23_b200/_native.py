@@ -93,6 +93,7 @@ SIGNATURES = {
     "tb_ntt_muladd6": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
     "tb_fft_muladd6": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
     "tb_set_lanes_per_cta": (ctypes.c_int, [_vp, ctypes.c_int]),
+    "tb_br6_lanes_per_cta": (ctypes.c_int, [_vp, ctypes.c_int64]),
     "tb_set_br_variant": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_set_ks_tile": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_set_narrow_lanes": (ctypes.c_int, [_vp, _i64]),

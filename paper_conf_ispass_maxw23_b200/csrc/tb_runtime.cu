@@ -59,7 +59,8 @@ static uint32_t brv10(uint32_t k) {
 
 struct tb_ctx {
     int device = 0;
-    int lanes_per_cta = 2;
+    int lanes_per_cta = 0;                  // br6 lanes per CTA (1..4), 0 = auto by wave quantisation (br6_lanes)
+    int sms = 0;                            // SM count (queried on first use)
     int variant = 6;                        // blind-rotation kernel: 6 = br6, 7 = br7 (TMA-staged BK), 8 = br8
     int ks_tile = 8;                        // gates per key-switch CTA (8, 16, 32); 8 measured fastest
     int narrow_lanes = 0;                   // launches with <= this many lanes run in latency mode (= SM count)
@@ -288,8 +289,27 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
     return TB_OK;
 }
 
+// Lanes per br6 CTA for a launch of `nlanes` lanes.  Fixed if set; auto picks 1 or 2 from the busiest SM's
+// lane count: G = 2 runs 2 CTAs (4 lanes) per SM at 2.79 ms per lane-slot, G = 1 runs 4 CTAs per SM at 2.96 ms
+// (profiles/r01f_lanes_sweep.txt: 592 / 1024 / 1536 / 2048 lanes).  A full wave favours G = 2 by 6 %, but G = 1
+// schedules the ragged last wave lane by lane instead of pair by pair (1,024 lanes: 20.5 vs 21.9 ms).
+static int br6_lanes(tb_ctx* c, int64_t nlanes) {
+    if (c->lanes_per_cta > 0) return c->lanes_per_cta;
+    if (c->sms == 0 && cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess)
+        c->sms = 148;
+    const int64_t s = c->sms;
+    const int64_t t1 = 296 * ((nlanes + s - 1) / s);              // busiest SM: lanes x 2.96 ms (x100)
+    const int64_t t2 = 2 * 279 * ((nlanes + 2 * s - 1) / (2 * s)); // busiest SM: 2 x CTAs x 2.79 ms (x100)
+    return t1 < t2 ? 1 : 2;
+}
+
+extern "C" int tb_br6_lanes_per_cta(tb_ctx* c, int64_t nlanes) {
+    if (!c || nlanes < 0) return fail(TB_EINVAL, "null context or negative lane count");
+    return br6_lanes(c, nlanes);
+}
+
 extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
-    if (!c || lanes < 1 || lanes > 4) return fail(TB_EINVAL, "lanes per CTA must be 1..4");
+    if (!c || lanes < 0 || lanes > 4) return fail(TB_EINVAL, "lanes per CTA must be 0 (auto) or 1..4");
     c->lanes_per_cta = lanes;
     return TB_OK;
 }
@@ -425,11 +445,11 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     else if (c->variant == 7)
         rc = launch_br7(A, 2, st);
     else if (c->variant == 10)
-        rc = launch_brf(A, std::min(std::max(c->lanes_per_cta, 1), 3), c->bkf, c->fftB, c->fftC, st);
+        rc = launch_brf(A, c->lanes_per_cta ? std::min(c->lanes_per_cta, 3) : 2, c->bkf, c->fftB, c->fftC, st);
     else if (c->variant == 8)
         rc = launch_br8(A, st);
     else
-        rc = launch_br6(A, c->lanes_per_cta, st);
+        rc = launch_br6(A, br6_lanes(c, nlanes), st);
     prof_end(c, slot, st);
     if (rc) return fail(TB_ECUDA, "blind-rotation kernel attribute/launch failed");
     cudaError_t e = cudaGetLastError();

@@ -214,8 +214,22 @@ def test_lanes_per_cta_and_ragged_tail(tb, ctx, keys, lanes):
         out = ctx.to_host(ctx.gates(tb.XOR, ctx.to_device(ca, 640), ctx.to_device(cb, 640)))
         assert (out == O.gates(keys, O.XOR, ca, cb)).all()
     finally:
-        ctx.set_lanes_per_cta(2)
+        ctx.set_lanes_per_cta(0)
         ctx.set_narrow_lanes(148)
+
+
+def test_auto_lanes_per_cta(tb, ctx):
+    """Auto lanes per CTA: 2 on full waves of 148 SMs x 4 lanes, 1 where lane-by-lane
+    scheduling of the ragged last wave wins (profiles/r01f_lanes_sweep.txt); fixed settings pass through."""
+    ctx.set_lanes_per_cta(0)
+    assert [ctx.br6_lanes_per_cta(n) for n in (592, 1024, 1536, 2048, 65536)] == [2, 1, 1, 2, 2]
+    ctx.set_lanes_per_cta(3)
+    try:
+        assert ctx.br6_lanes_per_cta(1024) == 3
+    finally:
+        ctx.set_lanes_per_cta(0)
+    with pytest.raises(tb.TBError):
+        ctx.set_lanes_per_cta(5)
 
 
 @pytest.mark.parametrize("lanes", [1, 2, 3])
@@ -230,7 +244,7 @@ def test_fft_variant_lanes_per_cta(tb, ctx, keys, lanes):
         got = ctx.bootstrap_wo_ks(ctx.to_device(cts))[:, :1025].cpu().numpy().view(np.uint32)
     finally:
         ctx.set_br_variant(6)
-        ctx.set_lanes_per_cta(2)
+        ctx.set_lanes_per_cta(0)
         ctx.set_narrow_lanes(148)
     for k in range(7):
         assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), k
