@@ -1,6 +1,6 @@
 """Narrow-level latency of each latency-mode kernel: device time of one level of L NAND gates (BR + KS).
 
-  python tools/latency.py [kernels...]     (default: 9 11)
+  python tools/latency.py [kernels...]     (default: 9 11; 6 = the throughput kernel br6, latency mode off)
 Inputs are seeded uniform words (evaluation is data-oblivious); parity is tests/test_gpu_parity.py's job.
 """
 import json
@@ -21,8 +21,11 @@ def main():
     g = torch.Generator(device=ctx.device)
     g.manual_seed(3)
     for k in kernels:
-        ctx.set_narrow_kernel(k)
-        for lanes in (1, 4, 16, 32, 37, 74, 148):
+        if k == 6:
+            ctx.set_narrow_lanes(0)
+        else:
+            ctx.set_narrow_kernel(k)
+        for lanes in (1, 4, 16, 32, 37, 74, 100, 148) + ((200, 296, 400, 592) if k == 6 else ()):
             a, b = ctx.empty(lanes), ctx.empty(lanes)
             a.random_(-2 ** 31, 2 ** 31 - 1, generator=g)
             b.random_(-2 ** 31, 2 ** 31 - 1, generator=g)
