@@ -153,6 +153,53 @@ def run_reference(args, rank):
     }), flush=True)
 
 
+# ------------------------------------------------------------------------------------------------ launch
+def _free_port():
+    import socket
+    so = socket.socket()
+    so.bind(("127.0.0.1", 0))
+    port = so.getsockname()[1]
+    so.close()
+    return port
+
+
+def spawn_ranks(args):
+    """`python bench.py --gpus N` without torchrun: start N ranks (one per GPU) ourselves, the way the driver
+    does (torch.distributed.run, rendezvous on 127.0.0.1).  Fails loudly if the node has fewer GPUs (a run that
+    silently timed one GPU would print the wrong n_gpus)."""
+    import torch
+    if not args.one_gpu_ranks:
+        have = torch.cuda.device_count()
+        if have < args.gpus:
+            print("bench.py: --gpus %d but only %d GPU(s) are visible on this node (use --one-gpu-ranks for a "
+                  "functional check of the N > 1 path on one GPU)" % (args.gpus, have), file=sys.stderr)
+            sys.exit(2)
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", str(args.gpus),
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+    sys.exit(subprocess.call(cmd))
+
+
+# ------------------------------------------------------------------------------------------------ latency roof
+# One bootstrap in latency mode runs on one cluster of the latency kernel (DESIGN.md "Latency roofline").  Its
+# floor is the pipe work of the 630 CMux steps spread over the cluster's SMs: brl (11) is FP64-bound, per CMux
+# step 6 forward + 4 inverse folded 512-point complex transforms (9 radix-2 stages x 256 butterflies, 6 FP64
+# lane-ops per CT and 8 per GS butterfly) + the MAC (6 rows x 4 outputs x 512 complex x 4 DFMA):
+#   6 x 13,824 + 4 x 18,432 + 49,152 = 205,824 FP64 lane-ops per CMux step, over 4 SMs x 64 FP64 lanes/clk.
+# br9 (9) is IMAD-bound: 12 transforms x 5,120 Shoup butterflies x 4 IMAD slots + 36,864 MACs x 2 + 6,144
+# reductions x 5 = 350,208 IMAD slots per step over 2 SMs x 64 IMAD lanes/clk.
+LATENCY_WORK = {11: ("brl_kernel", 205824, 4, "FP64 lane-ops"), 9: ("br9_kernel", 350208, 2, "IMAD slots")}
+
+
+def latency_roofline(level_ms, ks_ms, clk_mhz, kernel):
+    name, work, sms, unit = LATENCY_WORK[kernel]
+    floor_ms = N_LWE * work / (sms * 64 * clk_mhz * 1e6) * 1e3
+    br_ms = level_ms - ks_ms
+    return {"kernel": name, "cluster_sms": sms, "work_per_cmux": work, "unit": unit,
+            "floor_ms_630_steps": floor_ms, "measured_br_ms": br_ms, "frac": floor_ms / br_ms if br_ms > 0 else None,
+            "peak_source": "derived: %d SMs x 64 lanes/clk x %.0f MHz (median SM clock in the timed region)"
+                           % (sms, clk_mhz)}
+
+
 # ------------------------------------------------------------------------------------------------ ours
 def main():
     ap = argparse.ArgumentParser()
@@ -161,7 +208,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--gates-per-gpu", type=int, default=65536)
     ap.add_argument("--lanes-per-cta", type=int, default=0, help="0 = auto per launch size")
-    ap.add_argument("--br-variant", type=int, default=6, choices=[6, 7, 8, 10])
+    ap.add_argument("--br-variant", type=int, default=6, choices=[6, 10])
     ap.add_argument("--ks-tile", type=int, default=8, choices=[8, 16, 32])
     ap.add_argument("--exchange", default="fused", choices=["fused", "allgather"],
                     help="N > 1: per-level exchange of output rows (fused into the key switch over NVLink peer "
@@ -179,8 +226,16 @@ def main():
     if args.impl == "reference":
         run_reference(args, rank)
         return
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        spawn_ranks(args)
+    if world != args.gpus:
+        print("bench.py: --gpus %d but WORLD_SIZE=%d" % (args.gpus, world), file=sys.stderr)
+        sys.exit(2)
     if args.warmup < 3:
         args.warmup = 3                                  # timing rule: >= 3 warm-up steps
+    if world > 1:
+        os.environ.setdefault("NCCL_DEBUG", "INFO")     # keep the communicator / NVLS lines visible (stderr)
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
 
     import numpy as np
     import torch
@@ -200,11 +255,25 @@ def main():
         else:
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         group = dist.group.WORLD
+
+    def max_over_ranks(x):
+        if group is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=ctx.device)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sum_over_ranks(x):
+        if group is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=ctx.device)
+        dist.all_reduce(t)
+        return float(t.item())
+
     G = args.gates_per_gpu
     total = G * world
     ctx = tb.Context(local)
     ctx.set_lanes_per_cta(args.lanes_per_cta)
-    lpc = ctx.br6_lanes_per_cta(G)   # NAND/XOR level: one lane per gate
     ctx.set_br_variant(args.br_variant)
     ctx.set_ks_tile(args.ks_tile)
     ctx.load_keys(synth.random_words(tb.BK_WORDS, 11), synth.random_words(tb.KSK_WORDS, 12))
@@ -250,13 +319,10 @@ def main():
     ms = ev0.elapsed_time(ev1)
     br_ms, br_n, ks_ms, ks_n = ctx.profile_read()
     ctx.profile(False)
-    if group is not None:
-        t = torch.tensor([ms], device=ctx.device)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+    ms = max_over_ranks(ms)
     value = total * args.steps / (ms / 1e3)
 
-    # roofline of the dominant kernel (blind rotation).  Integer variants (br6/7/8): the integer-multiply
+    # roofline of the dominant kernel (blind rotation).  Integer variant (br6): the integer-multiply
     # (FMA-heavy) pipe.  Algorithmic work = IMAD issue slots of the method's modular arithmetic (DESIGN.md
     # "Roofline"): per CMux step 61,440 Shoup mulmods x 4 slots (IMAD + IMAD.HI(2) + IMAD) + 36,864 64-bit MACs
     # x 2 (IMAD.WIDE) + 6,144 MAC reductions x 5.  Peak = 148 SMs x 64 IMAD lanes/clk (fma pipe: 16
@@ -270,6 +336,8 @@ def main():
     sm_count = torch.cuda.get_device_properties(local).multi_processor_count
     clk_mhz = clocks.get("sm_mhz") or 1965.0
     peak = sm_count * 64 * clk_mhz * 1e6
+    throughput_launch = lanes_per_launch > sm_count      # launches of <= SM-count lanes run a latency kernel
+    lpc = ctx.br6_lanes_per_cta(lanes_per_launch) if args.br_variant == 6 and throughput_launch else None
     if args.br_variant == 10:
         per_bootstrap = N_LWE * CMUX_FP64_INSTR * 32
         unit, pipe = "G FP64-lane-ops/s", "FP64"
@@ -305,14 +373,28 @@ def main():
     if args.br_variant != 10:
         roofline["microbench_crosscheck"] = {"butterflies_per_s": bfly_rate, "macs_per_s": mac_rate,
                                              "frac_of_microbench": bfly_work / br_launch_s / bfly_rate}
+    # NTT-field choice (R1) from measured rates: per-bootstrap ceiling of each field's CMux work
+    fr = ctx.microbench_fields()
+    cmux30 = CMUX_BFLY / fr["shoup30_bfly_per_s"] + CMUX_MAC / fr["mac64_per_s"]
+    gl_mac = 2 * 6 * 1024 / fr["goldilocks_bfly_per_s"]          # 12,288 Goldilocks MAC mulmods ~ butterflies
+    cmux_gl = 8 * 5120 / fr["goldilocks_bfly_per_s"] + gl_mac
+    cmux_gl4 = 8 * (5120 / fr["goldilocks_shift_bfly_per_s"] + 992 / fr["goldilocks_bfly_per_s"]) + gl_mac
+    roofline["field_choice"] = dict(fr, **{
+        "bootstraps_per_s_ceiling_30bit_3part": 1 / (N_LWE * cmux30),
+        "bootstraps_per_s_ceiling_goldilocks_radix2": 1 / (N_LWE * cmux_gl),
+        "bootstraps_per_s_ceiling_goldilocks_fourstep": 1 / (N_LWE * cmux_gl4),
+        "note": "chip-wide register-resident rates; 30-bit: 12 transforms + 36,864 MACs per CMux; Goldilocks: 8 "
+                "transforms (radix-2, or four-step with 5,120 shift butterflies + 992 general twiddles each) + "
+                "12,288 MAC mulmods"})
 
-    # narrow-level latency (one gate)
-    lat = None
+    # narrow-level latency (one gate) and its roofline
     one = ctx.empty(2)
     one.random_(-2 ** 31, 2 ** 31 - 1, generator=gen)
     outl = ctx.empty(1)
     for _ in range(2):
         ctx.gates(tb.NAND, one[:1], one[1:2], out=outl)
+    torch.cuda.synchronize()
+    ctx.profile(True)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record()
     for _ in range(3):
@@ -320,37 +402,83 @@ def main():
     e1.record()
     torch.cuda.synchronize()
     lat = e0.elapsed_time(e1) / 3
+    _, _, lks_ms, lks_n = ctx.profile_read()
+    ctx.profile(False)
+    lat_roof = latency_roofline(lat, lks_ms / max(lks_n, 1), clk_mhz, 11)
 
-    # e2e through the C ABI with host buffers (per-rank replica of the per-GPU workload)
+    # e2e through the public API with host buffers: N = 1 the C ABI's tb_run_netlist_host; N > 1 the sharded
+    # level loop (each rank copies in the input rows its gates read, runs its shard with the level exchange,
+    # copies back the outputs it produced)
     e2e = None
     if not args.no_e2e:
-        nr = synth.independent_level(G, seed=15)
-        rnet = ctx.upload(tb.Netlist(nr["n_inputs"], nr["type"], nr["in0"], nr["in1"], nr["in2"]))
-        hin = torch.empty((nr["n_inputs"], tb.CT_WORDS), dtype=torch.int32, pin_memory=True)
-        hin.random_(-2 ** 31, 2 ** 31 - 1)
-        hout = torch.empty((G, tb.CT_WORDS), dtype=torch.int32, pin_memory=True)
-        ow = np.ascontiguousarray(nr["outputs"], np.int64)
-        ctx.run_netlist_host_into(rnet, hin, ow, hout)
-        if group is not None:
-            dist.barrier()
-        t0 = time.perf_counter()
-        for _ in range(args.steps):
+        if group is None:
+            nr = synth.independent_level(G, seed=15)
+            rnet = ctx.upload(tb.Netlist(nr["n_inputs"], nr["type"], nr["in0"], nr["in1"], nr["in2"]))
+            hin = torch.empty((nr["n_inputs"], tb.CT_WORDS), dtype=torch.int32, pin_memory=True)
+            hin.random_(-2 ** 31, 2 ** 31 - 1)
+            hout = torch.empty((G, tb.CT_WORDS), dtype=torch.int32, pin_memory=True)
+            ow = np.ascontiguousarray(nr["outputs"], np.int64)
             ctx.run_netlist_host_into(rnet, hin, ow, hout)
-        dt = time.perf_counter() - t0
-        if group is not None:
-            t = torch.tensor([dt], device=ctx.device, dtype=torch.float64)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            dt = float(t.item())
-        e2e = {"value": G * world * args.steps / dt, "unit": UNIT,
-               "h2d_bytes_per_step": int(nr["n_inputs"] * tb.CT_WORDS * 4),
-               "d2h_bytes_per_step": int(G * tb.CT_WORDS * 4),
-               "api": "tb_run_netlist_host (pinned host inputs -> device, run, outputs -> host, per rank)"}
-        rnet.free()
+            t0 = time.perf_counter()
+            for _ in range(args.steps):
+                ctx.run_netlist_host_into(rnet, hin, ow, hout)
+            dt = time.perf_counter() - t0
+            h2d, d2h = int(nr["n_inputs"] * tb.CT_WORDS * 4), int(G * tb.CT_WORDS * 4)
+            api = "tb_run_netlist_host (pinned host inputs -> device, all levels, outputs -> host)"
+            rnet.free()
+        else:
+            ow = np.ascontiguousarray(n["outputs"], np.int64)
+            in_rows, outs = ctx.shard_io(dnet, world, rank, ow)
+            r0 = int(in_rows[0]) if in_rows.size else 0
+            hin = torch.empty((max(int(in_rows[-1]) + 1 - r0, 1) if in_rows.size else 1, tb.WIRE_STRIDE),
+                              dtype=torch.int32, pin_memory=True)
+            hin.random_(-2 ** 31, 2 ** 31 - 1)
+            p0 = outs[0][0] if outs else 0
+            hout = torch.empty((max(outs[-1][0] + 1 - p0, 1) if outs else 1, tb.CT_WORDS), dtype=torch.int32,
+                               pin_memory=True)
+            run_e2e = lambda: ctx.run_netlist_host_sharded(dnet, hin, ow, hout, wires, group, exchange=exchange,
+                                                           inputs_row0=r0, out_pos0=p0)   # noqa: E731
+            run_e2e()
+            dist.barrier()
+            t0 = time.perf_counter()
+            for _ in range(args.steps):
+                h2d, d2h = run_e2e()
+            dt = time.perf_counter() - t0
+            h2d, d2h = int(sum_over_ranks(h2d)), int(sum_over_ranks(d2h))
+            api = ("Context.run_netlist_host_sharded (per rank: pinned host input rows of its shard -> device, "
+                   "sharded level loop with the %s exchange, its output rows -> host)" % exchange)
+        dt = max_over_ranks(dt)
+        e2e = {"value": total * args.steps / dt, "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "api": api}
+
+    # N > 1: the same level without the exchange step (each rank runs its own gate range; no peer stores, no
+    # barrier or all-gather inside the loop), to report the exchange's share of the level time
+    exch = None
+    if group is not None:
+        if exchange == "fused":
+            ctx.detach_peers()
+        dist.barrier()
+        torch.cuda.synchronize()
+        k2 = min(args.steps, 3)
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        f0.record()
+        for _ in range(k2):
+            for L, (row0, ng, _, _) in enumerate(dnet.levels, start=1):
+                a, b, _ = tb.parallel.shard(ng, world, rank)
+                if b > a:
+                    ctx.run_level(dnet, L, a, b, wires)
+        f1.record()
+        torch.cuda.synchronize()
+        no_ms = max_over_ranks(f0.elapsed_time(f1) / k2)
+        exch = {"level_ms_with_exchange": ms / args.steps, "level_ms_without_exchange": no_ms,
+                "exchange_share": 1.0 - no_ms / (ms / args.steps)}
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and not args.no_cpu_baseline:
         v, cores, sample = oracle_rate(n["type"])
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
+    if group is not None:
+        dist.barrier()                                    # other ranks wait while rank 0 times the oracle
 
     if rank == 0:
         print(json.dumps({
@@ -365,9 +493,10 @@ def main():
                        "exchange": exchange if world > 1 else None,
                        "lanes_per_cta": lpc, "br_variant": args.br_variant,
                        "l2": "inputs larger than L2 (%.0f MB of input ciphertexts per GPU)" % (2 * G * 2524 / 1e6)},
-            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+            "roofline": roofline, "latency_roofline": lat_roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
             "gpu_launches": br_n + ks_n,
             "latency_ms": {"level_of_%d_gates" % total: ms / args.steps, "level_of_1_gate": lat},
+            "exchange": exch,
         }), flush=True)
     if group is not None:
         dist.barrier()

@@ -186,10 +186,8 @@ int tb_fft_muladd6(tb_ctx* ctx, const int32_t* digits, const uint32_t* polys, ui
 int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
 /* The lanes per CTA the default kernel uses for a launch of `nlanes` lanes (>= 1), or < 0 (TB_EINVAL). */
 int tb_br6_lanes_per_cta(tb_ctx* ctx, int64_t nlanes);
-/* Blind-rotation kernel: 6 = br6_kernel (default: 6 warps/lane, 2 CTAs/SM, BK words from L2), 8 = br8_kernel
- * (two ping-ponged lane groups per CTA), 10 = brf_kernel (FP64-pipe FFT), 7 = br7_kernel
- * (2 lanes/CTA, 1 CTA/SM, each 144 KB BK step TMA-bulk-copied into shared memory one step ahead).  Both are
- * bit-identical; see DESIGN.md "Kernels". */
+/* Blind-rotation kernel: 6 = br6_kernel (default: 6 warps/lane, 2 CTAs/SM, BK words from L2), 10 = brf_kernel
+ * (FP64-pipe FFT).  Both are bit-identical; see DESIGN.md "Kernels".  Anything else: TB_EINVAL. */
 int tb_set_br_variant(tb_ctx* ctx, int variant);
 /* Latency mode for narrow levels: a launch with <= `lanes` bootstraps runs a latency-mode kernel (below)
  * instead of the throughput kernel.  Default = the device's SM count; 0 disables. */
@@ -198,8 +196,7 @@ int tb_set_narrow_lanes(tb_ctx* ctx, int64_t lanes);
  * else br9), 11 = brl_kernel (one bootstrap per cluster of 4 SMs on the FP64 path: each SM owns one output
  * polynomial and one 16-bit BK half, transforms split over warp pairs; 1.9 ms per level on B200),
  * 9 = br9_kernel (one bootstrap per cluster of 2 SMs, each SM owning one accumulator polynomial, forward-NTT
- * rows exchanged through distributed shared memory; 2.8 ms, 74 per wave), 7 = br7<1> (one bootstrap per SM).  All are
- * bit-identical.  Anything else: TB_EINVAL. */
+ * rows exchanged through distributed shared memory; 2.8 ms, 74 per wave).  Both are bit-identical.  Anything else: TB_EINVAL. */
 int tb_set_narrow_kernel(tb_ctx* ctx, int kernel);
 /* Level schedule used by tb_netlist_upload: Algorithm 1 gives every gate its earliest level;
  * with lanes > 0 gates that have slack are moved to later levels (never past their latest level, so the number
@@ -217,6 +214,11 @@ int tb_key_bytes(const tb_ctx* ctx, size_t* bytes);
  * butterfly, register resident, on all SMs for `iters` iterations; returns butterflies/s and the 64-bit
  * multiply-accumulate rate (MAC/s) measured with CUDA events.  Synchronous. */
 int tb_microbench(tb_ctx* ctx, int iters, double* butterflies_per_s, double* macs_per_s);
+/* Field microbenchmark behind the NTT-field choice (R1; the north star proposed the 64-bit Goldilocks
+ * prime): register-resident rates on all SMs, written to rates[0..3] = 30-bit Shoup butterflies/s (the kernels'
+ * own), Goldilocks general-twiddle butterflies/s, Goldilocks shift-twiddle (x 2^s) butterflies/s, 64-bit
+ * MACs/s.  Synchronous; iters <= 0 or null pointers: TB_EINVAL. */
+int tb_microbench_fields(tb_ctx* ctx, int iters, double* rates);
 
 const char* tb_last_error(void);
 const char* tb_version(void);

@@ -20,8 +20,21 @@ from dataclasses import dataclass
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SO = os.path.join(_HERE, "liboracle.so")
 _SRC = os.path.join(_HERE, "tfhe_oracle.c")
+
+
+def _cpu_tag() -> str:
+    """short hash of this host's CPU flags: the library is compiled with -march=native, so each host (this
+    container, the GPU box's host) gets its own build, compiled on first use"""
+    import hashlib
+    try:
+        flags = next(l for l in open("/proc/cpuinfo") if l.startswith("flags"))
+    except Exception:
+        flags = "unknown"
+    return hashlib.sha1(flags.encode()).hexdigest()[:10]
+
+
+_SO = os.path.join(_HERE, "liboracle-%s.so" % _cpu_tag())
 
 # gate codes: truth table f(a,b) at bit (2a+b) (C15); MUX = 3-input extension
 NOR, ANDNY, NOT, ANDYN, XOR, NAND, AND, XNOR, ORNY, ORYN, OR, MUX = 1, 2, 3, 4, 6, 7, 8, 9, 11, 13, 14, 16
@@ -31,12 +44,12 @@ GATE_NAMES = {NOR: "NOR", ANDNY: "ANDNY", NOT: "NOT", ANDYN: "ANDYN", XOR: "XOR"
 
 
 def build(force: bool = False) -> str:
-    """Compile liboracle.so with gcc (plain C + OpenMP).  -march=x86-64-v3 so the binary built here also
-    runs on the GPU box's host (the .so travels with the repo snapshot)."""
+    """Compile liboracle-<cpu>.so with gcc (plain C + OpenMP) at -O3 -march=native: one build per
+    host CPU type, so the cpu_baseline is not understated on a host with wider vector units."""
     if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < max(
             os.path.getmtime(_SRC), os.path.getmtime(os.path.join(_HERE, "tfhe_oracle.h"))):
         tmp = _SO + ".tmp%d" % os.getpid()
-        subprocess.check_call(["gcc", "-O3", "-march=x86-64-v3", "-fopenmp", "-fPIC", "-shared", "-std=c11",
+        subprocess.check_call(["gcc", "-O3", "-march=native", "-fopenmp", "-fPIC", "-shared", "-std=c11",
                                "-Wall", "-o", tmp, _SRC, "-lm"])
         os.replace(tmp, _SO)
     return _SO

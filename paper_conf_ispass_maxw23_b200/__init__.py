@@ -41,6 +41,11 @@ def version() -> str:
     return _native.lib().tb_version().decode()
 
 
+def _nullcontext():
+    import contextlib
+    return contextlib.nullcontext()
+
+
 def _ptr(t):
     return None if t is None else ctypes.c_void_p(t.data_ptr())
 
@@ -127,7 +132,7 @@ class Context:
         return rc
 
     def set_br_variant(self, variant: int):
-        """6 = br6_kernel (default), 7 = br7_kernel (TMA-staged BK); bit-identical outputs."""
+        """6 = br6_kernel (default), 10 = brf_kernel (FP64 pipe); bit-identical outputs."""
         _native.check(_native.lib().tb_set_br_variant(self._h, variant))
 
     def set_narrow_lanes(self, lanes: int):
@@ -139,7 +144,7 @@ class Context:
         _native.check(_native.lib().tb_set_level_capacity(self._h, lanes))
 
     def set_narrow_kernel(self, kernel: int):
-        """latency-mode kernel: 0 = auto (default), 11 = brl (4-SM cluster), 9 = br9 (2-SM cluster), 7 = br7<1>"""
+        """latency-mode kernel: 0 = auto (default), 11 = brl (4-SM cluster), 9 = br9 (2-SM cluster)"""
         _native.check(_native.lib().tb_set_narrow_kernel(self._h, kernel))
 
     def set_ks_tile(self, gates: int):
@@ -217,6 +222,13 @@ class Context:
         _native.check(_native.lib().tb_microbench(self._h, iters, ctypes.byref(b), ctypes.byref(m)))
         return b.value, m.value
 
+    def microbench_fields(self, iters: int = 4096) -> dict:
+        """measured butterfly / MAC rates of the 30-bit field and of Goldilocks (tb_microbench_fields)"""
+        r = (ctypes.c_double * 4)()
+        _native.check(_native.lib().tb_microbench_fields(self._h, iters, r))
+        return {"shoup30_bfly_per_s": r[0], "goldilocks_bfly_per_s": r[1], "goldilocks_shift_bfly_per_s": r[2],
+                "mac64_per_s": r[3]}
+
     def key_bytes(self) -> int:
         v = ctypes.c_size_t()
         _native.check(_native.lib().tb_key_bytes(self._h, ctypes.byref(v)))
@@ -251,9 +263,10 @@ class Context:
         run = lambda L, g0, g1: self.run_level(dnet, L, g0, g1, wires, stream)   # noqa: E731
         if exchange == "fused":
             self.attach_peers(wires, group)
-            parallel.level_loop(levels, wires, run, group, fused=True)
-        else:
-            parallel.level_loop(levels, wires, run, group)
+        # the per-level barrier / all-gather must be ordered on the stream the level kernels run on: make it the
+        # current stream for the loop (collectives order against torch's current stream)
+        with torch.cuda.stream(stream) if stream is not None else _nullcontext():
+            parallel.level_loop(levels, wires, run, group, fused=exchange == "fused")
 
     # ---- fused all-gather: the other ranks' wire arrays mapped into this process (CUDA IPC) ----
     def attach_peers(self, wires: torch.Tensor, group):
@@ -335,6 +348,73 @@ class Context:
                                                         output_wires.size, ctypes.c_void_p(out.data_ptr()),
                                                         out.stride(0)))
 
+    # ---- end to end over a process group (sharded level loop with host buffers) ----
+    def shard_io(self, dnet: DevNetlist, world: int, rank: int, output_wires=None):
+        """I/O plan of rank `rank` of the sharded level loop (parallel.shard per level): the input rows its gate
+        ranges read, and the (position in output_wires, wire row) pairs its gate ranges produce.  Host logic."""
+        key = (world, rank, None if output_wires is None else np.asarray(output_wires, np.int64).tobytes())
+        cache = dnet.__dict__.setdefault("_shard_io", {})
+        if key in cache:
+            return cache[key]
+        net, ni = dnet.net, dnet.net.n_inputs
+        order = np.argsort(dnet.row_of_wire[ni:], kind="stable")     # level-sorted position -> gate index
+        mine = []
+        for row0, ng, _, _ in dnet.levels:
+            g0, g1, _ = parallel.shard(ng, world, rank)
+            if g1 > g0:
+                mine.append(np.arange(row0 - ni + g0, row0 - ni + g1))
+        pos = np.concatenate(mine) if mine else np.zeros(0, np.int64)
+        g = order[pos]
+        ins = np.concatenate([net.in0[g], net.in1[g], net.in2[g]])
+        in_rows = np.unique(ins[(ins >= 0) & (ins < ni)])
+        outs = []
+        if output_wires is not None:
+            ow = np.asarray(output_wires, np.int64)
+            rows = dnet.row_of_wire[ow]
+            produced = np.zeros(dnet.n_rows, bool)
+            produced[ni + pos] = True
+            k = np.nonzero(produced[rows])[0]
+            outs = list(zip(k.tolist(), rows[k].tolist()))
+        cache[key] = (in_rows, outs)
+        return cache[key]
+
+    @staticmethod
+    def _runs(a, b=None):
+        """maximal runs where a (and b) advance by one together: [(a0, b0, length)]"""
+        a = np.asarray(a, np.int64)
+        b = a if b is None else np.asarray(b, np.int64)
+        if a.size == 0:
+            return []
+        brk = np.nonzero((np.diff(a) != 1) | (np.diff(b) != 1))[0] + 1
+        starts = np.concatenate([[0], brk])
+        ends = np.concatenate([brk, [a.size]])
+        return [(int(a[s]), int(b[s]), int(e - s)) for s, e in zip(starts, ends)]
+
+    def run_netlist_host_sharded(self, dnet: DevNetlist, inputs: torch.Tensor, output_wires, out: torch.Tensor,
+                                 wires: torch.Tensor, group, exchange: str = "fused", stream=None,
+                                 inputs_row0: int = 0, out_pos0: int = 0):
+        """End to end over a process group: this rank copies the input rows its gates read from host `inputs`
+        (pinned int32 rows; inputs[k] = input row inputs_row0 + k) into `wires`, runs the sharded level loop
+        (run_netlist with the group), copies the output rows its own gate ranges produced into `out` (pinned
+        int32 rows; out[k] = output_wires[out_pos0 + k]) and synchronises.  Together the ranks return every
+        output exactly once.  Returns (h2d_bytes, d2h_bytes) of this rank."""
+        in_rows, outs = self.shard_io(dnet, dist_world(group), dist_rank(group), output_wires)
+        if in_rows.size and (in_rows[0] < inputs_row0 or in_rows[-1] >= inputs_row0 + inputs.shape[0]):
+            raise ValueError("host inputs do not cover the input rows this rank reads")
+        if outs and (outs[0][0] < out_pos0 or outs[-1][0] >= out_pos0 + out.shape[0]):
+            raise ValueError("host output buffer does not cover the outputs this rank produces")
+        st = torch.cuda.current_stream(self.device) if stream is None else stream
+        w = inputs.shape[1]
+        with torch.cuda.stream(st):
+            for a, _, n in self._runs(in_rows):
+                wires[a:a + n, :w].copy_(inputs[a - inputs_row0:a - inputs_row0 + n], non_blocking=True)
+        self.run_netlist(dnet, wires, group, stream=st, exchange=exchange)
+        with torch.cuda.stream(st):
+            for k, r, n in self._runs([k for k, _ in outs], [r for _, r in outs]):
+                out[k - out_pos0:k - out_pos0 + n].copy_(wires[r:r + n, :out.shape[1]], non_blocking=True)
+        st.synchronize()
+        return int(in_rows.size) * w * 4, len(outs) * out.shape[1] * 4
+
     # ---- per-kernel device time (CUDA events around each launch) ----
     def profile(self, enable: bool):
         _native.check(_native.lib().tb_profile_enable(self._h, 1 if enable else 0))
@@ -360,6 +440,16 @@ class Context:
             self.close()
         except Exception:
             pass
+
+
+def dist_world(group) -> int:
+    import torch.distributed as dist
+    return dist.get_world_size(group) if group is not None else 1
+
+
+def dist_rank(group) -> int:
+    import torch.distributed as dist
+    return dist.get_rank(group) if group is not None else 0
 
 
 def slack_rows(dnet: DevNetlist, world: int) -> int:

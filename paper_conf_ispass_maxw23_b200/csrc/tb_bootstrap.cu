@@ -1,5 +1,5 @@
 // tb_bootstrap.cu -- load-time BK -> NTT-domain conversion and the tb_gates descriptor builder.
-// (The blind-rotation kernels themselves are in tb_br6.cu / tb_br7.cu.)
+// (The blind-rotation kernels themselves are in tb_br6.cu, tb_br9.cu, tb_brf.cu, tb_brl.cu.)
 //
 // The BK split used by every blind-rotation kernel: each torus coefficient
 // x = x0 + 2^11 x1 + 2^22 x2 (mod 2^32) with |x_m| <= 2^10, each part NTT-transformed mod p and pre-scaled by

@@ -165,12 +165,7 @@ __global__ void __launch_bounds__(192 * G, (G <= 2 ? 2 : 1)) br6_kernel(BrArgs A
 template <int G>
 static int launch_br6_g(const BrArgs& A, cudaStream_t st) {
     const size_t smem = sizeof(Br6Smem<G>);
-    static bool attr = false;
-    if (!attr) {
-        if (cudaFuncSetAttribute(br6_kernel<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
-            return -1;
-        attr = true;
-    }
+    if (ensure_smem_attr<br6_kernel<G>>(smem)) return -1;
     const int blocks = (A.nlanes + G - 1) / G;
     if (blocks == 0) return 0;
     br6_kernel<G><<<blocks, 192 * G, smem, st>>>(A);

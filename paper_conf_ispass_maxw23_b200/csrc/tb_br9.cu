@@ -1,7 +1,7 @@
 // tb_br9.cu -- latency-mode blind rotation: one bootstrap per thread-block cluster of two SMs (SURVEY 8(a)
 // rows a1-a5; SURVEY 8(f) f4 "split one gate's CMux across a thread-block cluster").
 //
-// Same arithmetic as br6/br7 (bit-identical).  CTA c of the cluster owns accumulator polynomial c (c = 0: a,
+// Same arithmetic as br6 (bit-identical).  CTA c of the cluster owns accumulator polynomial c (c = 0: a,
 // c = 1: b).  Per CMux step i:
 //   A  warps 0-2: digit jd of (X^abar - 1) ACC[c] -> forward NTT -> local rows (global rows r = 3c + jd); one
 //      thread pushes the 3 rows (12 KB) into the peer's receive buffer with a shared::cta -> shared::cluster
@@ -239,12 +239,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kB9Threads, 1) br9_k
 
 int launch_br9(const BrArgs& A, cudaStream_t st) {
     const size_t smem = sizeof(Br9Smem);
-    static bool attr = false;
-    if (!attr) {
-        if (cudaFuncSetAttribute(br9_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
-            return -1;
-        attr = true;
-    }
+    if (ensure_smem_attr<br9_kernel>(smem)) return -1;
     if (A.nlanes <= 0) return 0;
     br9_kernel<<<2 * A.nlanes, kB9Threads, smem, st>>>(A);
     return 0;

@@ -269,12 +269,7 @@ static int launch_brf_g(const BrArgs& A, const double2* bkf, const double2* twB,
     const size_t smem = sizeof(BrfSmem<G>);
     static_assert(sizeof(BrfSmem<G>) <= 232448, "brf shared memory");
     auto* kern = brf_kernel<G>;
-    static bool attr = false;
-    if (!attr) {
-        if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
-            return -1;
-        attr = true;
-    }
+    if (ensure_smem_attr<brf_kernel<G>>(smem)) return -1;
     const int blocks = (A.nlanes + G - 1) / G;
     if (blocks == 0) return 0;
     kern<<<blocks, BrfCfg<G>::NT, smem, st>>>(A, bkf, twB, twC);

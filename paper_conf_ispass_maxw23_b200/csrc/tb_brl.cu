@@ -359,13 +359,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
 }
 
 static int brl_attr() {
-    static bool attr = false;
-    if (!attr) {
-        if (cudaFuncSetAttribute(brl_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(BrlSmem)) !=
-            cudaSuccess)
-            return -1;
-        attr = true;
-    }
+    if (ensure_smem_attr<brl_kernel>(sizeof(BrlSmem))) return -1;
     return 0;
 }
 

@@ -139,6 +139,108 @@ __global__ void __launch_bounds__(256) mb_mac_kernel(uint64_t* sink, int iters, 
     if (s == 0x123456789ull) sink[blockIdx.x * blockDim.x + threadIdx.x] = s;
 }
 
+// ---- Goldilocks field p = 2^64 - 2^32 + 1 (the north star's proposed NTT field; R1) -----------
+// Register-resident butterflies over the 64-bit field, so that the field choice (30-bit Shoup field with the BK
+// split in 3 parts vs Goldilocks with 8 transforms per CMux) rests on measured rates of this GPU, not on
+// pipe-rate arithmetic.  Lazy representation in [0, 2^64); 2^64 = 2^32 - 1 and 2^96 = -1 (mod p).
+__device__ __forceinline__ uint64_t gl_red128(uint64_t lo, uint64_t hi) {
+    const uint32_t hl = (uint32_t)hi, hh = (uint32_t)(hi >> 32);
+    uint64_t t0 = lo - hh;
+    if (lo < hh) t0 -= 0xFFFFFFFFull;                    // borrow of 2^64 = 2^32 - 1
+    const uint64_t t1 = ((uint64_t)hl << 32) - hl;       // hl (2^32 - 1)
+    uint64_t r = t0 + t1;
+    if (r < t1) r += 0xFFFFFFFFull;                      // carry of 2^64
+    return r;
+}
+__device__ __forceinline__ uint64_t gl_add(uint64_t x, uint64_t y) {
+    uint64_t r = x + y;
+    if (r < x) r += 0xFFFFFFFFull;
+    return r;
+}
+__device__ __forceinline__ uint64_t gl_sub(uint64_t x, uint64_t y) {
+    uint64_t r = x - y;
+    if (x < y) r -= 0xFFFFFFFFull;
+    return r;
+}
+// CT butterfly with a general twiddle w (64 x 64 -> 128-bit product, then the reduction above)
+__device__ __forceinline__ void gl_bfly(uint64_t& x, uint64_t& y, uint64_t w) {
+    const uint64_t t = gl_red128(y * w, __umul64hi(y, w));
+    const uint64_t x0 = x;
+    x = gl_add(x0, t);
+    y = gl_sub(x0, t);
+}
+// CT butterfly whose twiddle is 2^s, 0 < s < 32 (four-step NTT with psi^32 = 8: shift-only inner/outer DFTs)
+__device__ __forceinline__ void gl_bfly_shift(uint64_t& x, uint64_t& y, int s) {
+    const uint64_t t = gl_red128(y << s, y >> (64 - s));
+    const uint64_t x0 = x;
+    x = gl_add(x0, t);
+    y = gl_sub(x0, t);
+}
+template <int NV, bool SHIFT>
+__global__ void __launch_bounds__(256) mb_gl_kernel(uint64_t* sink, int iters, uint64_t w, int sh) {
+    uint64_t x[NV], y[NV];
+#pragma unroll
+    for (int i = 0; i < NV; i++) {
+        x[i] = threadIdx.x * 0x9E3779B97F4A7C15ull + i;
+        y[i] = threadIdx.x * 0xC2B2AE3D27D4EB4Full + 3u * i;
+    }
+    for (int it = 0; it < iters; it++) {
+#pragma unroll
+        for (int i = 0; i < NV; i++) {
+            if (SHIFT) gl_bfly_shift(x[i], y[i], sh);
+            else gl_bfly(x[i], y[i], w);
+        }
+        w ^= (uint64_t)(it & 1);
+        sh = (sh & 15) + 3;
+    }
+    uint64_t s = 0;
+#pragma unroll
+    for (int i = 0; i < NV; i++) s += x[i] ^ y[i];
+    if (s == 0x123456789ull) sink[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+
+// rates[0] = 30-bit Shoup butterflies/s (the kernels' own), [1] Goldilocks general-twiddle butterflies/s,
+// [2] Goldilocks shift-twiddle butterflies/s, [3] 64-bit MACs/s; all SMs, register resident
+int run_microbench_fields(int iters, double* rates) {
+    double b = 0, m = 0;
+    if (run_microbench(iters, &b, &m)) return -1;
+    int dev = 0, sms = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return -1;
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return -1;
+    const int blocks = sms * 8, threads = 256;
+    void* sink = nullptr;
+    if (cudaMalloc(&sink, (size_t)blocks * threads * 8) != cudaSuccess) return -1;
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    float best_g = 1e30f, best_s = 1e30f;
+    for (int rep = 0; rep < 4; rep++) {
+        float ms = 0;
+        cudaEventRecord(e0);
+        mb_gl_kernel<8, false><<<blocks, threads>>>((uint64_t*)sink, iters, 0x61E96455F799F0A0ull, 3);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (rep > 0) best_g = ms < best_g ? ms : best_g;
+        cudaEventRecord(e0);
+        mb_gl_kernel<8, true><<<blocks, threads>>>((uint64_t*)sink, iters, 0ull, 3);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (rep > 0) best_s = ms < best_s ? ms : best_s;
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(sink);
+    if (cudaGetLastError() != cudaSuccess) return -1;
+    const double ops = (double)blocks * threads * iters * 8.0;
+    rates[0] = b;
+    rates[1] = ops / (best_g * 1e-3);
+    rates[2] = ops / (best_s * 1e-3);
+    rates[3] = m;
+    return 0;
+}
+
 int run_microbench(int iters, double* bfly, double* mac) {
     int dev = 0, sms = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) return -1;

@@ -2,9 +2,25 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <atomic>
+
 #include "tb_common.cuh"
 
 namespace tb {
+
+// The >48 KB dynamic shared-memory opt-in (cudaFuncSetAttribute) is per device: remembered per (kernel, device)
+// so that contexts on several GPUs of one process each get it (one atomic bit per device).
+template <auto Kern>
+inline int ensure_smem_attr(size_t bytes) {
+    static std::atomic<uint64_t> done{0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return -1;
+    const uint64_t bit = 1ull << (dev & 63);
+    if (done.load(std::memory_order_acquire) & bit) return 0;
+    if (cudaFuncSetAttribute(Kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes) != cudaSuccess) return -1;
+    done.fetch_or(bit, std::memory_order_acq_rel);
+    return 0;
+}
 
 // blind rotation + extraction over a batch of lanes (tb_bootstrap.cu)
 struct BrArgs {
@@ -40,8 +56,6 @@ struct KsArgs {
 };
 
 int launch_br6(const BrArgs& A, int G, cudaStream_t st);
-int launch_br7(const BrArgs& A, int G, cudaStream_t st);
-int launch_br8(const BrArgs& A, cudaStream_t st);
 int launch_br9(const BrArgs& A, cudaStream_t st);
 void launch_bk_to_ntt(const uint32_t* bk, uint32_t* bkhat, const uint2* twF, uint32_t ninv, uint32_t ninvp,
                       cudaStream_t st);
@@ -57,6 +71,7 @@ int set_ntt_constants(const uint32_t* fw, const uint32_t* fwp, const uint32_t* i
 int launch_ntt_muladd6(const int32_t* digits, const uint32_t* polys, uint32_t* res, const uint2* twF,
                        const uint2* twI, uint32_t ninv, uint32_t ninvp, cudaStream_t st);
 int run_microbench(int iters, double* bfly, double* mac);
+int run_microbench_fields(int iters, double* rates);
 
 }  // namespace tb
 

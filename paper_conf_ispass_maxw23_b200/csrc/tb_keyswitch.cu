@@ -210,12 +210,7 @@ __global__ void ksk_relayout_kernel(const uint32_t* __restrict__ src, uint32_t* 
 template <int T>
 static int launch_ks_t(const KsArgs& A, uint32_t* partial, int S, cudaStream_t st) {
     const size_t smem = (size_t)kN * T * 2 + T * 4;
-    static bool attr = false;
-    if (!attr) {
-        if (cudaFuncSetAttribute(ks_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
-            return -1;
-        attr = true;
-    }
+    if (ensure_smem_attr<ks_kernel<T>>(smem)) return -1;
     const int blocks = (A.ngates + T - 1) / T;
     ks_kernel<T><<<dim3(blocks, S), kKsThreads, smem, st>>>(A, S > 1 ? partial : nullptr, S);
     if (S > 1) ks_reduce_kernel<<<A.ngates, kKsThreads, 0, st>>>(A, partial, S);

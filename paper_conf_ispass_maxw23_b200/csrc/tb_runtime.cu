@@ -61,10 +61,10 @@ struct tb_ctx {
     int device = 0;
     int lanes_per_cta = 0;                  // br6 lanes per CTA (1..4), 0 = auto by wave quantisation (br6_lanes)
     int sms = 0;                            // SM count (queried on first use)
-    int variant = 6;                        // blind-rotation kernel: 6 = br6, 7 = br7 (TMA-staged BK), 8 = br8
+    int variant = 6;                        // blind-rotation kernel: 6 = br6, 10 = brf (FP64 pipe)
     int ks_tile = 8;                        // gates per key-switch CTA (8, 16, 32); 8 measured fastest
     int narrow_lanes = 0;                   // launches with <= this many lanes run in latency mode (= SM count)
-    int narrow_kernel = 0;                  // latency-mode kernel: 9 = br9 (2-SM cluster per lane), 7 = br7<1>,
+    int narrow_kernel = 0;                  // latency-mode kernel: 9 = br9 (2-SM cluster per lane),
                                             // 11 = brl (4-SM cluster per lane, FP64 path), 0 = auto:
                                             // brl while the lanes fit in one wave of its clusters, else br9
     int brl_wave = -2;                      // co-resident brl clusters (queried on first use)
@@ -290,16 +290,20 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
 }
 
 // Lanes per br6 CTA for a launch of `nlanes` lanes.  Fixed if set; auto picks 1 or 2 from the busiest SM's
-// lane count: G = 2 runs 2 CTAs (4 lanes) per SM at 2.79 ms per lane-slot, G = 1 runs 4 CTAs per SM at 2.96 ms
-// (profiles/r01f_lanes_sweep.txt: 592 / 1024 / 1536 / 2048 lanes).  A full wave favours G = 2 by 6 %, but G = 1
-// schedules the ragged last wave lane by lane instead of pair by pair (1,024 lanes: 20.5 vs 21.9 ms).
+// lane count.  This is a CALIBRATION, not a model: the per-lane-slot times below were measured on a 148-SM
+// B200 by tools/lanes_sweep.sh (profiles/r01f_lanes_sweep.txt: 592 / 1024 / 1536 / 2048 lanes x G = 1..4) and
+// must be re-measured whenever br6_kernel changes.  G = 2 runs 2 CTAs (4 lanes) per SM at kBr6SlotG2 per
+// lane-slot, G = 1 runs 4 CTAs per SM at kBr6SlotG1.  A full wave favours G = 2 by 6 %, but G = 1 schedules the
+// ragged last wave lane by lane instead of pair by pair (1,024 lanes: 20.5 vs 21.9 ms).
+constexpr int64_t kBr6SlotG1 = 296;   // ms x 100 per 630-step lane slot, G = 1 (4 CTAs/SM)
+constexpr int64_t kBr6SlotG2 = 279;   // ms x 100 per lane slot, G = 2 (2 CTAs/SM)
 static int br6_lanes(tb_ctx* c, int64_t nlanes) {
     if (c->lanes_per_cta > 0) return c->lanes_per_cta;
     if (c->sms == 0 && cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess)
         c->sms = 148;
     const int64_t s = c->sms;
-    const int64_t t1 = 296 * ((nlanes + s - 1) / s);              // busiest SM: lanes x 2.96 ms (x100)
-    const int64_t t2 = 2 * 279 * ((nlanes + 2 * s - 1) / (2 * s)); // busiest SM: 2 x CTAs x 2.79 ms (x100)
+    const int64_t t1 = kBr6SlotG1 * ((nlanes + s - 1) / s);              // busiest SM: lanes x slot time
+    const int64_t t2 = 2 * kBr6SlotG2 * ((nlanes + 2 * s - 1) / (2 * s)); // busiest SM: 2 x CTAs x slot time
     return t1 < t2 ? 1 : 2;
 }
 
@@ -315,15 +319,15 @@ extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
 }
 
 extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
-    if (!c || !(variant == 6 || variant == 7 || variant == 8 || variant == 10))
-        return fail(TB_EINVAL, "blind-rotation variant must be 6, 7, 8 or 10");
+    if (!c || !(variant == 6 || variant == 10))
+        return fail(TB_EINVAL, "blind-rotation variant must be 6 or 10");
     c->variant = variant;
     return TB_OK;
 }
 
 extern "C" int tb_set_narrow_kernel(tb_ctx* c, int kernel) {
-    if (!c || (kernel != 0 && kernel != 7 && kernel != 9 && kernel != 11))
-        return fail(TB_EINVAL, "latency-mode kernel must be 0 (auto), 7, 9 or 11");
+    if (!c || (kernel != 0 && kernel != 9 && kernel != 11))
+        return fail(TB_EINVAL, "latency-mode kernel must be 0 (auto), 9 or 11");
     c->narrow_kernel = kernel;
     return TB_OK;
 }
@@ -439,15 +443,10 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
         nk = nlanes <= c->brl_wave ? 11 : 9;
     }
     if (c->narrow_lanes > 0 && nlanes <= c->narrow_lanes)
-        rc = nk == 9    ? launch_br9(A, st)                    // narrow level: one lane per 2-SM cluster
-             : nk == 11 ? launch_brl(A, c->bkf, c->fftL, st)   // or per 4-SM cluster (FP64)
-                                      : launch_br7(A, 1, st);                // or one lane per SM
-    else if (c->variant == 7)
-        rc = launch_br7(A, 2, st);
+        rc = nk == 9 ? launch_br9(A, st)                       // narrow level: one lane per 2-SM cluster
+                     : launch_brl(A, c->bkf, c->fftL, st);     // or per 4-SM cluster (FP64)
     else if (c->variant == 10)
         rc = launch_brf(A, c->lanes_per_cta ? std::min(c->lanes_per_cta, 3) : 2, c->bkf, c->fftB, c->fftC, st);
-    else if (c->variant == 8)
-        rc = launch_br8(A, st);
     else
         rc = launch_br6(A, br6_lanes(c, nlanes), st);
     prof_end(c, slot, st);
@@ -469,7 +468,8 @@ static int run_ks(tb_ctx* c, const uint32_t* lanes, int64_t lane_base, int64_t l
     const bool split = c->narrow_lanes > 0 && ngates <= c->narrow_lanes;   // narrow level: split each gate's KS
     // mid-size level: tiles sliced over the input coefficients so that the launch still fills the GPU
     const int slices = split ? 1 : ks_tile_slices(ngates, c->ks_tile);
-    const size_t need = split ? ks_split_scratch_words(std::max<int64_t>(ngates, c->narrow_lanes))
+    // the split launch writes ngates x ks_split_count(ngates) partial rows (the slice count falls as ngates grows)
+    const size_t need = split ? ks_split_scratch_words(ngates)
                               : (slices > 1 ? (size_t)ngates * slices * kKsRow : 0);
     if (need > c->ks_scratch_words) {
         cudaFree(c->ks_scratch);
@@ -596,6 +596,13 @@ extern "C" int tb_microbench(tb_ctx* c, int iters, double* bfly, double* mac) {
     if (!c || !bfly || !mac || iters <= 0) return fail(TB_EINVAL, "bad argument");
     TB_CUDA(cudaSetDevice(c->device));
     if (run_microbench(iters, bfly, mac)) return fail(TB_ECUDA, "microbenchmark failed");
+    return TB_OK;
+}
+
+extern "C" int tb_microbench_fields(tb_ctx* c, int iters, double* rates) {
+    if (!c || !rates || iters <= 0) return fail(TB_EINVAL, "bad argument");
+    TB_CUDA(cudaSetDevice(c->device));
+    if (run_microbench_fields(iters, rates)) return fail(TB_ECUDA, "microbenchmark failed");
     return TB_OK;
 }
 

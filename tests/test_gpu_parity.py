@@ -89,26 +89,33 @@ def test_bootstrap_wo_ks_bit_exact(tb, ctx, keys):
         assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), k
 
 
-@pytest.mark.parametrize("kernel", [0, 9, 7, 11])
+def oracle_bootstrap_many(keys, cts):
+    """O.bootstrap_wo_ks over independent rows on all host cores (ctypes releases the GIL)"""
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(O.max_threads()) as ex:
+        return np.stack(list(ex.map(lambda c: O.bootstrap_wo_ks(keys, c), cts)))
+
+
+@pytest.mark.parametrize("kernel", [0, 9, 11])
 def test_narrow_level_latency_mode_bit_exact(tb, ctx, keys, kernel):
-    """small launches run the latency kernel (br9: 2-SM cluster per lane, br7<1>: one SM per lane, brl: 4-SM
-    cluster per lane on the FP64 path; 40 lanes = 160 CTAs is more than one wave); 149 lanes fall back to the
-    throughput kernel"""
+    """small launches run the latency kernel (br9: 2-SM cluster per lane, brl: 4-SM cluster per lane on the
+    FP64 path; 40 lanes = 160 CTAs is more than one wave of brl); 149 lanes fall back to the throughput kernel.
+    Every lane of the 1-, 3- and 40-lane launches is compared with the oracle, the first and last of 149."""
     rng = np.random.default_rng(39 + kernel)
     ctx.set_narrow_kernel(kernel)
     try:
         for count in (1, 3, 40, 149):
             cts = rng.integers(0, M32, (count, 631), dtype=np.uint64).astype(np.uint32)
             got = ctx.bootstrap_wo_ks(ctx.to_device(cts))[:, :1025].cpu().numpy().view(np.uint32)
-            for k in sorted({0, count - 1}):
-                assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all(), (count, k)
+            idx = np.arange(count) if count <= 40 else np.array([0, count - 1])
+            assert (got[idx] == oracle_bootstrap_many(keys, cts[idx])).all(), count
     finally:
         ctx.set_narrow_kernel(0)
 
 
-@pytest.mark.parametrize("variant", [6, 7, 8, 10])
+@pytest.mark.parametrize("variant", [6, 10])
 def test_blind_rotation_variants_bit_exact(tb, ctx, keys, variant):
-    """every blind-rotation kernel variant (br6 / br7 TMA-staged / br8 ping-pong) on a ragged batch of 9"""
+    """every blind-rotation kernel variant (br6 integer NTT / brf FP64 FFT) on a ragged batch of 9"""
     rng = np.random.default_rng(40 + variant)
     cts = rng.integers(0, M32, (9, 631), dtype=np.uint64).astype(np.uint32)
     ctx.set_br_variant(variant)
@@ -221,8 +228,17 @@ def test_lanes_per_cta_and_ragged_tail(tb, ctx, keys, lanes):
 def test_auto_lanes_per_cta(tb, ctx):
     """Auto lanes per CTA: 2 on full waves of 148 SMs x 4 lanes, 1 where lane-by-lane
     scheduling of the ragged last wave wins (profiles/r01f_lanes_sweep.txt); fixed settings pass through."""
+    import torch
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    slot1, slot2 = 296, 279             # the calibration constants of tb_runtime.cu (kBr6SlotG1 / kBr6SlotG2)
+
+    def expect(n):                      # busiest-SM estimate on this device's SM count
+        return 1 if slot1 * -(-n // sms) < 2 * slot2 * -(-n // (2 * sms)) else 2
     ctx.set_lanes_per_cta(0)
-    assert [ctx.br6_lanes_per_cta(n) for n in (592, 1024, 1536, 2048, 65536)] == [2, 1, 1, 2, 2]
+    sizes = (4 * sms, 1024, 1536, 2048, 65536)
+    assert [ctx.br6_lanes_per_cta(n) for n in sizes] == [expect(n) for n in sizes]
+    if sms == 148:                      # the measured B200 picks (profiles/r01f_lanes_sweep.txt)
+        assert [ctx.br6_lanes_per_cta(n) for n in sizes] == [2, 1, 1, 2, 2]
     ctx.set_lanes_per_cta(3)
     try:
         assert ctx.br6_lanes_per_cta(1024) == 3

@@ -12,7 +12,9 @@ wrong rounding) in the step it covers fails it:
   * bootstrap (a2-a6, C6)   -- trivial input (0, phi) -> (0, +-mu) exactly, at the real parameters
   * blind rotation (a2-a5)  -- structured zero-noise key: phase = +-mu by the sign rule, exactly
   * gates (a1, a7)          -- truth tables after decryption, toy and real parameters
-  * noise                   -- [7]'s variance bounds for BR and KS at the real parameters
+  * decryption (C11)        -- exact phase-0 / int32 sign-edge ciphertexts built from the secret
+  * level executor          -- ripple-carry adder through or_level_batch: decrypted sum == a + b
+  * noise                   -- [7]'s variance bounds for BR (256 bootstraps) and KS at the real parameters
 Phases in these tests are computed in plain Python (brute force) so the check does not route through
 the oracle's own phase function.
 """
@@ -23,6 +25,7 @@ import numpy as np
 import pytest
 
 import oracle as O
+import synth
 
 M32 = 1 << 32
 MU = 1 << 29
@@ -306,26 +309,88 @@ def test_not_is_negation():
     assert ((out.astype(np.uint64) + c) % M32 == 0).all()
 
 
+# ---------------------------------------------------------------- decryption tie (C11) and netlists
+def test_decrypt_phase_zero_is_zero_and_sign_edges():
+    """C11: Decrypt = [(int32) phase > 0]; an exact phase-0 ciphertext decrypts to 0 (a `>= 0` slip fails here),
+    and the int32 sign edges: phase 1 -> 1, 2^31 - 1 -> 1, 2^31 (= -2^31) -> 0, 2^32 - 1 (= -1) -> 0"""
+    keys = O.keygen(O.TOY, seed=21, with_bk=False, with_ksk=False)
+    rng = np.random.default_rng(22)
+    phases = [0, 1, (1 << 31) - 1, 1 << 31, M32 - 1, MU, M32 - MU]
+    cts = np.zeros((len(phases), O.TOY.n + 1), np.uint32)
+    for k, ph in enumerate(phases):
+        a = rng.integers(0, M32, O.TOY.n, dtype=np.uint64)
+        cts[k, :O.TOY.n] = a
+        cts[k, O.TOY.n] = (ph + int((a * keys.s.astype(np.uint64)).sum())) % M32   # b = <a,s> + phase exactly
+    assert [py_lwe_phase(keys.s.tolist(), c.tolist()) for c in cts] == phases
+    assert O.decrypt_bits(keys, cts).tolist() == [0, 1, 1, 0, 0, 1, 0]
+
+
+def _rca_oracle(keys, bits_n, A, B, seed):
+    """Algorithm 1 levels of the ripple-carry adder, each evaluated by O.run_level (or_level_batch)"""
+    from oracle.algorithm1 import algorithm1
+    n = synth.ripple_carry_adder(bits_n)
+    x = np.concatenate([synth.pack_bits([A], bits_n), synth.pack_bits([B], bits_n)])
+    w = np.zeros((n["n_inputs"] + len(n["type"]), keys.params.n + 1), np.uint32)
+    w[:n["n_inputs"]] = O.encrypt_bits(keys, x, seed)
+    for batch in algorithm1(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"]):
+        b = np.array(batch)
+        O.run_level(keys, w, n["type"][b], n["in0"][b], n["in1"][b], n["in2"][b], n["n_inputs"] + b)
+    return int(synth.unpack_bits(O.decrypt_bits(keys, w[n["outputs"]]), bits_n + 1)[0])
+
+
+def test_level_batch_ripple_carry_adder_toy():
+    """or_level_batch (the oracle's level executor, used by the GPU parity tests) end to end on the 8-bit RCA of
+    cfg 2: the decrypted sum equals a + b for seeded pairs, edge pairs included"""
+    keys = O.keygen(O.TOY, seed=23)
+    rng = np.random.default_rng(24)
+    pairs = [(0, 0), (255, 255), (255, 1), (128, 128)] + [tuple(rng.integers(0, 256, 2)) for _ in range(4)]
+    for k, (A, B) in enumerate(pairs):
+        assert _rca_oracle(keys, 8, int(A), int(B), 30 + k) == int(A) + int(B), (A, B)
+
+
+@pytest.mark.slow
+def test_level_batch_ripple_carry_adder_real_params(real_keys):
+    """the same at the real parameters on a 2-bit adder (7 gates, 4 levels)"""
+    assert _rca_oracle(real_keys, 2, 3, 3, 40) == 6
+    assert _rca_oracle(real_keys, 2, 2, 1, 41) == 3
+
+
 # ---------------------------------------------------------------- noise bounds ([7]; SURVEY 8(c) noise row)
+def np_trlwe_phase_binary(S, acc, N):
+    """phase(b - a * S) of a TRLWE sample for a binary S in numpy: a * S = sum_{j: S_j = 1} X^j a (negacyclic
+    shifts), independent of the oracle's C code"""
+    a, b = acc[:N].astype(np.int64), acc[N:].astype(np.int64)
+    prod = np.zeros(N, np.int64)
+    for j in np.nonzero(S)[0]:
+        rot = np.concatenate([-a[N - j:], a[:N - j]])        # X^j a mod X^N + 1
+        prod = (prod + rot) % M32
+    return (b - prod) % M32
+
+
 @pytest.mark.slow
 def test_blind_rotation_noise_within_bound(real_keys):
-    """MSE of phase(ACC) - X^{-phibar} v over all N coefficients <= V_BR bound 1.408e-5 + 3.7e-8."""
+    """MSE of phase(ACC) - X^{-phibar} v over all N coefficients of 256 blind rotations <= V_BR bound
+    1.408e-5 + 3.7e-8 (the mean-square error, bias included, over >= 256 bootstraps)."""
+    from concurrent.futures import ThreadPoolExecutor
     P = O.DEFAULT
-    rng = random.Random(9)
+    K = 256
+    cts = O.encrypt_bits(real_keys, np.arange(K) & 1, 100)
+    with ThreadPoolExecutor(O.max_threads()) as ex:           # ctypes releases the GIL
+        accs = list(ex.map(lambda c: O.blind_rotate(real_keys, c), cts))
+    two_N = 2 * P.N
+    # tfhe-lib mod switch (pinned above): round(v 2N / 2^32) = ((v + 2^20) mod 2^32) >> 21
+    ms = lambda v: ((np.asarray(v, np.uint64) + (1 << 20)) % M32) >> 21
+    s = real_keys.s.astype(np.uint64)
     errs = []
-    for k in range(2):
-        ct = O.encrypt_bits(real_keys, [k & 1], 100 + k)[0]
-        acc = O.blind_rotate(real_keys, ct)
-        ph = py_trlwe_phase(real_keys.S.tolist(), acc.tolist())
-        two_N = 2 * P.N
-        ms = lambda v: O.mod_switch(int(v), two_N)
-        phibar = (ms(ct[P.n]) - sum(ms(ct[i]) * int(real_keys.s[i]) for i in range(P.n))) % two_N
+    for ct, acc in zip(cts, accs):
+        ph = np_trlwe_phase_binary(real_keys.S, acc, P.N)
+        phibar = (int(ms(ct[P.n])) - int((ms(ct[:P.n]) * s).sum())) % two_N
         # expected message: X^{-phibar} (mu,...,mu): coefficient c = +mu if c + phibar mod 2N < N else -mu
-        for c in range(P.N):
-            e = (c + phibar) % two_N
-            want = MU if e < P.N else M32 - MU
-            errs.append(signed(ph[c] - want) / M32)
-    mse = float(np.mean(np.square(errs)))
+        e = (np.arange(P.N) + phibar) % two_N
+        want = np.where(e < P.N, MU, M32 - MU)
+        d = (ph - want) % M32
+        errs.append(np.where(d >= 1 << 31, d - M32, d) / M32)
+    mse = float(np.mean(np.square(np.concatenate(errs))))
     assert mse < 1.408e-5 + 3.7e-8, mse
     assert mse > 1e-7            # the noise is really there (keys are not noiseless)
 

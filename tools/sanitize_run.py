@@ -32,13 +32,13 @@ if LAT:
     ok = torch.equal(res[0][:, :1025], res[1][:, :1025])
     print("latency kernels agree:", ok)
     sys.exit(0 if ok else 1)
-for variant in ((6,) if QUICK else (6, 7, 8, 10)):
+for variant in ((6,) if QUICK else (6, 10)):
     ctx.set_br_variant(variant)
     ctx.set_narrow_lanes(0)
     outs.append(ctx.bootstrap_wo_ks(ct))
 ctx.set_br_variant(6)
 ctx.set_narrow_lanes(148)
-for k in (() if QUICK else (11, 9, 7)):                      # latency mode: brl, br9, br7<1>
+for k in (() if QUICK else (11, 9)):                         # latency mode: brl, br9
     ctx.set_narrow_kernel(k)
     outs.append(ctx.bootstrap_wo_ks(ct))
 ctx.set_narrow_kernel(0)
