@@ -101,13 +101,22 @@ def gpu_id_for(dev: int) -> str:
 
 
 # ------------------------------------------------------------------------------------------------ oracle
+def host_threads():
+    """the host cores this process may use (torchrun sets OMP_NUM_THREADS=1 per rank; the oracle legs run on
+    rank 0 alone while the other ranks wait, so they take every core)"""
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
 def oracle_rate(G_types, seconds_hint=None):
     """Time the CPU oracle on a bounded sample of the workload: 4 gates per host thread (NAND/XOR as in
     the GPU arm) with real seeded keys; returns (gates/s, threads, sample description)."""
     import numpy as np
     import oracle as O
     import synth
-    threads = O.max_threads()
+    threads = host_threads()
     keys = O.keygen(O.DEFAULT, seed=99)
     ns = 4 * threads
     types = np.asarray(G_types[:ns], np.int32)
@@ -128,7 +137,7 @@ def run_reference(args, rank):
     import oracle as O
     import synth
     O.build()
-    threads = O.max_threads()
+    threads = host_threads()
     keys = O.keygen(O.DEFAULT, seed=99)
     n = synth.independent_level(threads * (args.warmup + args.steps), seed=1)
     bits = synth.random_bits(2 * n["type"].size, 2)
@@ -383,6 +392,7 @@ def main():
         "bootstraps_per_s_ceiling_30bit_3part": 1 / (N_LWE * cmux30),
         "bootstraps_per_s_ceiling_goldilocks_radix2": 1 / (N_LWE * cmux_gl),
         "bootstraps_per_s_ceiling_goldilocks_fourstep": 1 / (N_LWE * cmux_gl4),
+        "goldilocks_over_30bit_cmux_time": min(cmux_gl, cmux_gl4) / cmux30,
         "note": "chip-wide register-resident rates; 30-bit: 12 transforms + 36,864 MACs per CMux; Goldilocks: 8 "
                 "transforms (radix-2, or four-step with 5,120 shift butterflies + 992 general twiddles each) + "
                 "12,288 MAC mulmods"})

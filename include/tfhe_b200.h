@@ -219,6 +219,13 @@ int tb_microbench(tb_ctx* ctx, int iters, double* butterflies_per_s, double* mac
  * own), Goldilocks general-twiddle butterflies/s, Goldilocks shift-twiddle (x 2^s) butterflies/s, 64-bit
  * MACs/s.  Synchronous; iters <= 0 or null pointers: TB_EINVAL. */
 int tb_microbench_fields(tb_ctx* ctx, int iters, double* rates);
+/* Tensor-core check (diagnostic): D[128][N] = A[128][K] . B[N][K]^T as integers through tcgen05.mma kind::i8
+ * (device pointers; A bytes signed if a_signed else unsigned, likewise B; D s32), with the operand tiles laid
+ * out in shared memory as K-major core matrices whose K-adjacent stride is `lbo` bytes (the layout of the
+ * tensor-core NTT).  Synchronous.  K % 32, N % 16, K <= 256, N <= 256, lbo >= 128
+ * and lbo % 16 == 0, else TB_EINVAL. */
+int tb_tc_mma_test(tb_ctx* ctx, const uint8_t* A, const uint8_t* B, int K, int N, int a_signed, int b_signed,
+                   int lbo, int32_t* D);
 
 const char* tb_last_error(void);
 const char* tb_version(void);

@@ -229,6 +229,16 @@ class Context:
         return {"shoup30_bfly_per_s": r[0], "goldilocks_bfly_per_s": r[1], "goldilocks_shift_bfly_per_s": r[2],
                 "mac64_per_s": r[3]}
 
+    def tc_mma_test(self, A: np.ndarray, B: np.ndarray, a_signed: bool = False, b_signed: bool = False,
+                    lbo: int = 128) -> np.ndarray:
+        """diagnostic: A [128][K] . B [N][K]^T as s32 through tcgen05.mma kind::i8 (tb_tc_mma_test)"""
+        a = torch.from_numpy(np.ascontiguousarray(A).view(np.uint8)).to(self.device)
+        b = torch.from_numpy(np.ascontiguousarray(B).view(np.uint8)).to(self.device)
+        d = torch.empty((128, B.shape[0]), dtype=torch.int32, device=self.device)
+        _native.check(_native.lib().tb_tc_mma_test(self._h, _ptr(a), _ptr(b), A.shape[1], B.shape[0], int(a_signed),
+                                                   int(b_signed), lbo, _ptr(d)))
+        return d.cpu().numpy()
+
     def key_bytes(self) -> int:
         v = ctypes.c_size_t()
         _native.check(_native.lib().tb_key_bytes(self._h, ctypes.byref(v)))

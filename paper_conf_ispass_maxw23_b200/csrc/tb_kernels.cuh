@@ -72,6 +72,8 @@ int launch_ntt_muladd6(const int32_t* digits, const uint32_t* polys, uint32_t* r
                        const uint2* twI, uint32_t ninv, uint32_t ninvp, cudaStream_t st);
 int run_microbench(int iters, double* bfly, double* mac);
 int run_microbench_fields(int iters, double* rates);
+int run_tc_mma_test(const uint8_t* A, const uint8_t* B, int K, int N, int a_signed, int b_signed, int lbo, int32_t* D,
+                    cudaStream_t st);
 
 }  // namespace tb
 

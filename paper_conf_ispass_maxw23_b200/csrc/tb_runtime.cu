@@ -606,6 +606,18 @@ extern "C" int tb_microbench_fields(tb_ctx* c, int iters, double* rates) {
     return TB_OK;
 }
 
+extern "C" int tb_tc_mma_test(tb_ctx* c, const uint8_t* A, const uint8_t* B, int K, int N, int a_signed, int b_signed,
+                              int lbo, int32_t* D) {
+    if (!c || !A || !B || !D) return fail(TB_EINVAL, "null argument");
+    TB_CUDA(cudaSetDevice(c->device));
+    const int rc = run_tc_mma_test(A, B, K, N, a_signed, b_signed, lbo, D, c->own);
+    if (rc == -2) return fail(TB_EINVAL, "K must be a multiple of 32 <= 256, N a multiple of 16 <= 256, lbo >= 128");
+    if (rc) return fail(TB_ECUDA, "tensor-core test launch failed");
+    TB_CUDA(cudaGetLastError());
+    TB_CUDA(cudaStreamSynchronize(c->own));
+    return TB_OK;
+}
+
 // ------------------------------------------------------------------------------------------ netlists
 // Algorithm 1: starting from the inputs (ready = finished = I), each iteration computes every
 // node whose predecessors are all ready.  The iteration in which gate g first enters C - finished is

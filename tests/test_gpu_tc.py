@@ -1,0 +1,41 @@
+"""Tensor-core (tcgen05.mma kind::i8) building blocks against plain integer arithmetic (-m gpu).
+
+The tensor-core NTT of the blind rotation multiplies byte limbs on the tensor
+cores; these tests pin the descriptor encodings, operand layouts (K-major core matrices, padded strides), the
+s8 / u8 signedness and the TMEM read-back against numpy's exact int64 matrix product.
+"""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import paper_conf_ispass_maxw23_b200 as tb
+    tb.build()
+    c = tb.Context(0)
+    yield c
+    c.close()
+
+
+@pytest.mark.parametrize("K,N,a_signed,lbo", [(32, 16, False, 128), (32, 128, True, 144), (128, 128, False, 144),
+                                              (128, 128, True, 128), (256, 256, False, 144)])
+def test_mma_i8_equals_integer_matmul(ctx, K, N, a_signed, lbo):
+    rng = np.random.default_rng(K + N + lbo)
+    A = rng.integers(-128 if a_signed else 0, 128 if a_signed else 256, (128, K)).astype(np.int8 if a_signed else np.uint8)
+    B = rng.integers(0, 256, (N, K)).astype(np.uint8)
+    D = ctx.tc_mma_test(A, B, a_signed=a_signed, b_signed=False, lbo=lbo)
+    want = A.astype(np.int64) @ B.astype(np.int64).T
+    assert (D.astype(np.int64) == want).all()
+
+
+def test_mma_i8_extremes(ctx):
+    """all-255 x all-255 at K = 256: 256 * 255^2 = 16,646,400 per entry, the largest the NTT accumulates"""
+    A = np.full((128, 256), 255, np.uint8)
+    B = np.full((256, 256), 255, np.uint8)
+    D = ctx.tc_mma_test(A, B, lbo=144)
+    assert (D == 256 * 255 * 255).all()
