@@ -187,7 +187,8 @@ int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
 /* The lanes per CTA the default kernel uses for a launch of `nlanes` lanes (>= 1), or < 0 (TB_EINVAL). */
 int tb_br6_lanes_per_cta(tb_ctx* ctx, int64_t nlanes);
 /* Blind-rotation kernel: 6 = br6_kernel (default: 6 warps/lane, 2 CTAs/SM, BK words from L2), 10 = brf_kernel
- * (FP64-pipe FFT).  Both are bit-identical; see DESIGN.md "Kernels".  Anything else: TB_EINVAL. */
+ * (FP64-pipe FFT), 12 = brt_kernel (four-step NTT on the tcgen05 tensor cores, DESIGN.md
+ * "Tensor-core NTT").  All are bit-identical; see DESIGN.md "Kernels".  Anything else: TB_EINVAL. */
 int tb_set_br_variant(tb_ctx* ctx, int variant);
 /* Latency mode for narrow levels: a launch with <= `lanes` bootstraps runs a latency-mode kernel (below)
  * instead of the throughput kernel.  Default = the device's SM count; 0 disables. */
@@ -219,6 +220,12 @@ int tb_microbench(tb_ctx* ctx, int iters, double* butterflies_per_s, double* mac
  * own), Goldilocks general-twiddle butterflies/s, Goldilocks shift-twiddle (x 2^s) butterflies/s, 64-bit
  * MACs/s.  Synchronous; iters <= 0 or null pointers: TB_EINVAL. */
 int tb_microbench_fields(tb_ctx* ctx, int iters, double* rates);
+/* Tensor-core external-product core (diagnostic): for two lanes g and both output polynomials q,
+ * res[g][q][.] = sum_{r<6} digits[g][r] (x) polys[r][q] mod 2^32 (negacyclic), computed exactly as one CMux step
+ * of the tensor-core blind rotation does it (four-step NTT on tcgen05 kind::i8, MAC against the NTT-domain BK,
+ * inverse, centred lift).  Device pointers: digits int32 [2][6][1024] in [-64, 63],
+ * polys u32 [6][2][1024] (one BK_i), res u32 [2][2][1024].  Synchronous. */
+int tb_tc_muladd(tb_ctx* ctx, const int32_t* digits, const uint32_t* polys, uint32_t* res);
 /* Tensor-core check (diagnostic): D[128][N] = A[128][K] . B[N][K]^T as integers through tcgen05.mma kind::i8
  * (device pointers; A bytes signed if a_signed else unsigned, likewise B; D s32), with the operand tiles laid
  * out in shared memory as K-major core matrices whose K-adjacent stride is `lbo` bytes (the layout of the

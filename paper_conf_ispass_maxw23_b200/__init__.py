@@ -132,7 +132,7 @@ class Context:
         return rc
 
     def set_br_variant(self, variant: int):
-        """6 = br6_kernel (default), 10 = brf_kernel (FP64 pipe); bit-identical outputs."""
+        """6 = br6_kernel (default), 10 = brf_kernel (FP64 pipe), 12 = brt_kernel (tensor cores); bit-identical."""
         _native.check(_native.lib().tb_set_br_variant(self._h, variant))
 
     def set_narrow_lanes(self, lanes: int):
@@ -228,6 +228,13 @@ class Context:
         _native.check(_native.lib().tb_microbench_fields(self._h, iters, r))
         return {"shoup30_bfly_per_s": r[0], "goldilocks_bfly_per_s": r[1], "goldilocks_shift_bfly_per_s": r[2],
                 "mac64_per_s": r[3]}
+
+    def tc_muladd(self, digits: torch.Tensor, polys: torch.Tensor) -> torch.Tensor:
+        """diagnostic: [2][2][1024] = sum_r digits[g][r] (x) polys[r][q] through the tensor-core CMux (tb_tc_muladd)"""
+        res = torch.empty((2, 2, N_RING), dtype=torch.int32, device=self.device)
+        d, p = digits.contiguous(), polys.contiguous()
+        _native.check(_native.lib().tb_tc_muladd(self._h, _ptr(d), _ptr(p), _ptr(res)))
+        return res
 
     def tc_mma_test(self, A: np.ndarray, B: np.ndarray, a_signed: bool = False, b_signed: bool = False,
                     lbo: int = 128) -> np.ndarray:

@@ -103,6 +103,7 @@ SIGNATURES = {
     "tb_microbench_fields": (ctypes.c_int, [_vp, ctypes.c_int, ctypes.POINTER(ctypes.c_double)]),
     "tb_tc_mma_test": (ctypes.c_int, [_vp, _vp, _vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                       ctypes.c_int, _vp]),
+    "tb_tc_muladd": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
     "tb_microbench": (ctypes.c_int, [_vp, ctypes.c_int, ctypes.POINTER(ctypes.c_double),
                                      ctypes.POINTER(ctypes.c_double)]),
     "tb_last_error": (ctypes.c_char_p, []),

@@ -1,0 +1,501 @@
+// tb_brt.cu -- blind rotation on the 5th-generation tensor cores (DESIGN.md
+// "Tensor-core NTT").
+//
+// PAPER.md: bootstrapping "dominates the execution time", blind rotation is the largest slice of a gate
+// (Fig. 7) and its NTT work is "highly vectorizable".  The arithmetic is the same exact integer
+// external product as br6 (field p = 0x3FFF7801, BK split in 3 signed 11-bit parts, centred lift; DESIGN.md
+// "Exactness"), but each length-1024 negacyclic NTT is evaluated in four steps whose two 32-point DFTs are
+// integer matrix products on the tensor cores (tcgen05.mma kind::i8, byte limbs, s32 accumulators in TMEM):
+//
+//   forward   a[32 k1 + k2] -> B[j1][k2] = sum_k1 W1[j1][k1] a[32 k1 + k2]          W1 = psi^(32 (2 j1 + 1) k1)
+//             C[j1][k2] = B[j1][k2] psi^((2 j1 + 1) k2)                              (twiddle, CUDA cores)
+//             A[j1 + 32 j2] = sum_k2 W2[j2][k2] C[j1][k2]                            W2 = psi^(64 j2 k2)
+//   i.e. A[j] = a(psi^(2 j + 1)), the evaluation at the roots of X^1024 + 1 in natural order;
+//   inverse   D[j1][k2] = sum_j2 V2[k2][j2] M[j1 + 32 j2]                            V2 = psi^(-64 j2 k2)
+//             E[j1][k2] = D[j1][k2] psi^(-(2 j1 + 1) k2)
+//             N a[32 k1 + k2] = sum_j1 V1[k1][j1] E[j1][k2]                          V1 = psi^(-32 (2 j1 + 1) k1)
+//
+// A product with a 30-bit constant matrix is exact as sum_b 2^(8 b) (X . bytes_b(W)); a 30-bit data operand
+// enters as its 4 bytes along K, against bytes_b(2^(8 c) W mod p) (precomputed), so every GEMM is
+// u8 x u8 (digits: s8 x u8) with K = 32 (digits) or 128 and N = 128 (4 limbs x 32), and the CUDA cores only
+// recombine the 4 limbs (one Shoup product by 2^16) and apply the twiddles.
+//
+// A CTA = G = 2 lanes (bootstraps) = 12 polynomials per transform = three M = 128 tiles; one CTA per SM;
+// accumulators resident in shared memory for all n = 630 CMux steps; 12 warps, thread 0 issues the MMAs.
+#include <cstring>
+
+#include "tb_kernels.cuh"
+#include "tb_ntt.cuh"
+#include "tb_tc.cuh"
+
+namespace tb {
+
+constexpr int kTcG = 2;                       // lanes per CTA
+constexpr int kTcPolys = 6 * kTcG;            // polynomials per transform stage (12 = 3 tiles of 4)
+constexpr int kTcWarps = 12;
+constexpr int kTcThreads = 32 * kTcWarps;
+// shared-memory operand layouts (K-major core matrices, tb_tc.cuh)
+constexpr uint32_t kA1Lbo = 128, kA1Sbo = 256;          // digits: 384 rows x 32 B
+constexpr uint32_t kOpLbo = 144, kOpSbo = 8 * 144;      // 30-bit operands: 3 tiles x 128 rows x 128 B (padded)
+constexpr uint32_t kOpTile = 16 * kOpSbo;               // 18,432 B
+constexpr uint32_t kB1Bytes = 128 * 32, kBBytes = 128 * 128;
+constexpr uint32_t kTcBTotal = kB1Bytes + 3 * kBBytes;  // B1 (W1 bytes), B2 (W2'), B3 (V2'), B4 (V1')
+constexpr int kBk4Rec = 36;                              // NTT-domain BK record per coefficient: [r][o]
+
+struct BrtSmem {
+    unsigned char B[kTcBTotal];                  // constant B operands (dense: LBO 128)
+    unsigned char A1[kTcPolys * 32 * 32];        // digit operand
+    unsigned char op[3 * kOpTile];               // 30-bit operand / MAC buffer (A2, MAC in/out = A3, A4)
+    uint2 twF[32 * 32];                          // [j1][k2] (psi^((2 j1 + 1) k2), Shoup)
+    uint2 twI[32 * 32];                          // [k2][j1] (psi^(-(2 j1 + 1) k2), Shoup)
+    uint32_t acc[kTcG][2][kN];
+    uint16_t bar[kTcG][kn + 2];
+    uint64_t mbar;
+    uint32_t tmem;
+};
+
+// ---- limb recombination: sum_b 2^(8 b) Y_b mod p, result in [0, 4p) --------------------------------
+constexpr uint32_t kW16 = 1u << 16;
+constexpr uint32_t kW16p = (uint32_t)((((uint64_t)1 << 48)) / kP);    // Shoup companion of 2^16
+__device__ __forceinline__ uint32_t limbs_u(uint32_t y0, uint32_t y1, uint32_t y2, uint32_t y3) {
+    const uint32_t lo = y0 + (y1 << 8), hi = y2 + (y3 << 8);           // each < 2^31 + 2^23 < 4p
+    const uint32_t q = __umulhi(hi, kW16p);
+    const uint32_t r = (hi << 16) - q * kP;                            // hi 2^16 mod p in [0, 2p)
+    return red_2p(lo) + r;
+}
+__device__ __forceinline__ uint32_t limbs_s(uint32_t y0, uint32_t y1, uint32_t y2, uint32_t y3) {
+    // signed limbs (s8 digits x u8): |Y_b| < 2^19, so lo + p, hi + p are in (0, 2p)
+    const uint32_t lo = y0 + (y1 << 8) + kP, hi = y2 + (y3 << 8) + kP;
+    const uint32_t q = __umulhi(hi, kW16p);
+    const uint32_t r = (hi << 16) - q * kP;
+    return lo + r;
+}
+
+// ---- one GEMM stage: tiles x K-steps, one commit ------------------------------------------------------
+__device__ __forceinline__ void brt_gemm(const BrtSmem& S, uint32_t tmem, int stage) {
+    // stage 0: A1 x B1 (K = 32, s8 digits); 1: op x B2; 2: op x B3; 3: op (tile m) x B4 -> columns 128 m
+    const uint32_t sB = smem_u32(S.B), sA1 = smem_u32(S.A1), sOp = smem_u32(S.op);
+    if (stage == 0) {
+        constexpr uint32_t id = tc_idesc_i8(128, 128, true, false);
+        for (int t = 0; t < 3; t++)
+            tc_mma_i8(tmem + 128 * t, tc_sdesc(sA1 + t * 16 * kA1Sbo, kA1Lbo, kA1Sbo), tc_sdesc(sB, 128, 256), id, 0);
+    } else {
+        constexpr uint32_t id = tc_idesc_i8(128, 128, false, false);
+        const uint32_t bb = sB + kB1Bytes + (stage - 1) * kBBytes;
+        for (int t = 0; t < 3; t++)
+            for (int s = 0; s < 4; s++)
+                tc_mma_i8(tmem + 128 * t, tc_sdesc(sOp + t * kOpTile + 2 * s * kOpLbo, kOpLbo, kOpSbo),
+                          tc_sdesc(bb + 2 * s * 128, 128, 1024), id, s > 0);
+    }
+    tc_commit(smem_u32(&S.mbar));
+}
+
+__device__ __forceinline__ uint32_t op_word_off(int row, int word) { return tc_off(row, 4 * word, kOpLbo, kOpSbo); }
+
+// ---- the CMux pipeline after the digits are in A1 (shared by the kernel and the diagnostic) ----------
+// bk4: this step's NTT-domain BK records [32 j1 + j2][36]; out: ep4 result added into acc[g][q][.]
+__device__ __forceinline__ void brt_cmux_tail(BrtSmem& S, const uint32_t* __restrict__ bk4, uint32_t& phase) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t tq = S.tmem + ((uint32_t)(32 * (warp & 3)) << 16);   // this warp's TMEM lane quadrant
+    const int t = warp >> 2;                                           // tile of polynomial P = warp
+    const int P = warp;
+    // GEMM1: digits x W1
+    fence_async_smem();
+    tc_fence_before();
+    __syncthreads();
+    if (tid == 0) {
+        tc_fence_after();
+        brt_gemm(S, S.tmem, 0);
+    }
+    mbar_wait(&S.mbar, phase);
+    phase ^= 1;
+    tc_fence_after();
+    // ep1: thread (P, k2 = lane): B[j1][k2] -> C = B . psi^((2 j1 + 1) k2) -> op row (P, j1), word k2
+    {
+        const int k2 = lane;
+        for (int jc = 0; jc < 8; jc++) {
+            uint32_t v[16];
+            tc_ld16(tq + 128 * t + 16 * jc, v);
+            tc_wait_ld();
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const int j1 = 4 * jc + u;
+                const uint32_t x = limbs_s(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3]);
+                const uint2 w = S.twF[j1 * 32 + k2];
+                *reinterpret_cast<uint32_t*>(S.op + t * kOpTile + op_word_off((P & 3) * 32 + j1, k2)) =
+                    shoup_mul(x, w.x, w.y);
+            }
+        }
+    }
+    fence_async_smem();
+    tc_fence_before();
+    __syncthreads();
+    if (tid == 0) {
+        tc_fence_after();
+        brt_gemm(S, S.tmem, 1);
+    }
+    mbar_wait(&S.mbar, phase);
+    phase ^= 1;
+    tc_fence_after();
+    // ep2: thread (P, j1 = lane): A[j1 + 32 j2] for j2 = 4c..4c+3 -> [0, 2p) -> op row (P, j1), words 4c..4c+3
+    {
+        const int j1 = lane;
+        unsigned char* rowp = S.op + t * kOpTile;
+        for (int c = 0; c < 8; c++) {
+            uint32_t v[16];
+            tc_ld16(tq + 128 * t + 16 * c, v);
+            tc_wait_ld();
+            uint4 o;
+            o.x = red_2p(limbs_u(v[0], v[1], v[2], v[3]));
+            o.y = red_2p(limbs_u(v[4], v[5], v[6], v[7]));
+            o.z = red_2p(limbs_u(v[8], v[9], v[10], v[11]));
+            o.w = red_2p(limbs_u(v[12], v[13], v[14], v[15]));
+            *reinterpret_cast<uint4*>(rowp + op_word_off((P & 3) * 32 + j1, 4 * c)) = o;
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    // MAC: coefficient (j1, j2) of both lanes: M_o = sum_r A_r . BK4[r][o] (a4.3), in place (o reuses row r = o)
+    {
+        const uint32_t R = c_misc[0], Rp = c_misc[1];
+        for (int pos = tid; pos < kN; pos += kTcThreads) {
+            const int j1 = pos >> 5, j2 = pos & 31;
+            const uint4* rec = reinterpret_cast<const uint4*>(bk4 + (size_t)pos * kBk4Rec);
+            uint32_t B[kBk4Rec];
+#pragma unroll
+            for (int k = 0; k < kBk4Rec / 4; k++) {
+                const uint4 b4 = __ldg(rec + k);
+                B[4 * k] = b4.x; B[4 * k + 1] = b4.y; B[4 * k + 2] = b4.z; B[4 * k + 3] = b4.w;
+            }
+#pragma unroll
+            for (int g = 0; g < kTcG; g++) {
+                uint32_t* w[6];
+                uint32_t D[6];
+#pragma unroll
+                for (int r = 0; r < 6; r++) {
+                    const int PP = g * 6 + r;
+                    w[r] = reinterpret_cast<uint32_t*>(S.op + (PP >> 2) * kOpTile + op_word_off((PP & 3) * 32 + j1, j2));
+                    D[r] = *w[r];
+                }
+#pragma unroll
+                for (int o = 0; o < 6; o++) {
+                    uint64_t s = 0;
+#pragma unroll
+                    for (int r = 0; r < 6; r++) s += (uint64_t)D[r] * B[r * 6 + o];
+                    const uint32_t hi = (uint32_t)(s >> 32), lo = (uint32_t)s;
+                    *w[o] = red_2p(shoup_mul(hi, R, Rp) + (lo - (lo >> 30) * kP));
+                }
+            }
+        }
+    }
+    fence_async_smem();
+    tc_fence_before();
+    __syncthreads();
+    if (tid == 0) {
+        tc_fence_after();
+        brt_gemm(S, S.tmem, 2);
+    }
+    mbar_wait(&S.mbar, phase);
+    phase ^= 1;
+    tc_fence_after();
+    // ep3: thread (O = g*6 + o, j1 = lane): D[j1][k2] -> E = D . psi^(-(2 j1 + 1) k2) -> A4 tile m = o % 3,
+    // row (g*2 + q)*32 + k2, word j1
+    {
+        const int j1 = lane, O = P, g = O / 6, o = O % 6, q = o / 3, m = o % 3;
+        unsigned char* dst = S.op + m * kOpTile;   // GEMM3 has consumed op (A3): it is rewritten as A4
+        for (int c = 0; c < 8; c++) {
+            uint32_t v[16];
+            tc_ld16(tq + 128 * t + 16 * c, v);
+            tc_wait_ld();
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const int k2 = 4 * c + u;
+                const uint32_t x = limbs_u(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3]);
+                const uint2 w = S.twI[k2 * 32 + j1];
+                *reinterpret_cast<uint32_t*>(dst + op_word_off((g * 2 + q) * 32 + k2, j1)) = shoup_mul(x, w.x, w.y);
+            }
+        }
+    }
+    fence_async_smem();
+    tc_fence_before();
+    __syncthreads();
+    if (tid == 0) {
+        tc_fence_after();
+        const uint32_t sB4 = smem_u32(S.B) + kB1Bytes + 2 * kBBytes, sOp = smem_u32(S.op);
+        constexpr uint32_t id = tc_idesc_i8(128, 128, false, false);
+        for (int m = 0; m < 3; m++)
+            for (int s = 0; s < 4; s++)
+                tc_mma_i8(S.tmem + 128 * m, tc_sdesc(sOp + m * kOpTile + 2 * s * kOpLbo, kOpLbo, kOpSbo),
+                          tc_sdesc(sB4 + 2 * s * 128, 128, 1024), id, s > 0);
+        tc_commit(smem_u32(&S.mbar));
+    }
+    mbar_wait(&S.mbar, phase);
+    phase ^= 1;
+    tc_fence_after();
+    // ep4: thread (g, q, k2 = lane) [quadrant = g*2 + q]: the 3 parts of coefficient 32 k1 + k2 -> centred lift,
+    // << 11 m, summed into ACC (a4.4); the three warps of a quadrant split k1 in groups of 4
+    {
+        const int quad = warp & 3, g = quad >> 1, q = quad & 1, k2 = lane;
+        const int kg0 = (warp >> 2) * 3, kg1 = kg0 + 3 < 8 ? kg0 + 3 : 8;
+        for (int kg = kg0; kg < kg1; kg++) {
+            uint32_t v0[16], v1[16], v2[16];
+            tc_ld16(tq + 0 * 128 + 16 * kg, v0);
+            tc_ld16(tq + 1 * 128 + 16 * kg, v1);
+            tc_ld16(tq + 2 * 128 + 16 * kg, v2);
+            tc_wait_ld();
+#pragma unroll
+            for (int u = 0; u < 4; u++) {
+                const int k1 = 4 * kg + u;
+                const uint32_t a0 = lift_centred(red_2p(limbs_u(v0[4 * u], v0[4 * u + 1], v0[4 * u + 2], v0[4 * u + 3])));
+                const uint32_t a1 = lift_centred(red_2p(limbs_u(v1[4 * u], v1[4 * u + 1], v1[4 * u + 2], v1[4 * u + 3])));
+                const uint32_t a2 = lift_centred(red_2p(limbs_u(v2[4 * u], v2[4 * u + 1], v2[4 * u + 2], v2[4 * u + 3])));
+                uint32_t* acc = &S.acc[g][q][32 * k1 + k2];
+                *acc = *acc + a0 + (a1 << 11) + (a2 << 22);
+            }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+}
+
+// ---- digits of (X^abar - 1) ACC for both lanes -> A1 (a4.1) -----------------------------------------
+// task (g, bloc, k2, h): 16 coefficients c = 32 (16 h + i) + k2, three digit bytes each, one 16-B store per digit
+__device__ __forceinline__ void brt_digits(BrtSmem& S, int i) {
+    const int tid = threadIdx.x;
+    if (tid >= kTcG * 2 * 32 * 2) return;
+    const int k2 = tid & 31, h = (tid >> 5) & 1, bloc = (tid >> 6) & 1, g = tid >> 7;
+    const uint32_t ab = S.bar[g][i];
+    const uint32_t* acc = S.acc[g][bloc];
+    uint32_t d[3][4] = {};
+#pragma unroll
+    for (int u = 0; u < 16; u++) {
+        const uint32_t c = 32u * (16 * h + u) + k2;
+        const uint32_t mm = (c - ab) & (kTwoN - 1);
+        const uint32_t src = acc[mm & (kN - 1)];
+        const uint32_t rot = mm < (uint32_t)kN ? src : 0u - src;
+        const uint32_t x = rot - acc[c] + c_misc[3];             // (X^abar - 1) ACC + decomposition offset
+#pragma unroll
+        for (int jd = 0; jd < 3; jd++) {
+            const uint32_t dig = ((x >> (32 - kBgbit * (jd + 1))) & 127u) - 64u;   // digit in [-64, 63]
+            d[jd][u >> 2] |= (dig & 0xFFu) << (8 * (u & 3));
+        }
+    }
+#pragma unroll
+    for (int jd = 0; jd < 3; jd++) {
+        const int P = g * 6 + bloc * 3 + jd;
+        const uint32_t row = P * 32 + k2;
+        *reinterpret_cast<uint4*>(S.A1 + tc_off(row, 16 * h, kA1Lbo, kA1Sbo)) =
+            make_uint4(d[jd][0], d[jd][1], d[jd][2], d[jd][3]);
+    }
+}
+
+__device__ __forceinline__ void brt_setup(BrtSmem& S, const unsigned char* tcB, const uint2* tcTw) {
+    const int tid = threadIdx.x;
+    for (int k = tid; k < (int)(kTcBTotal / 16); k += kTcThreads)
+        reinterpret_cast<uint4*>(S.B)[k] = __ldg(reinterpret_cast<const uint4*>(tcB) + k);
+    for (int k = tid; k < 32 * 32; k += kTcThreads) {
+        S.twF[k] = tcTw[k];
+        S.twI[k] = tcTw[1024 + k];
+    }
+    if (tid < 32) tc_alloc<512>(&S.tmem);
+    if (tid == 0) {
+        mbar_init(&S.mbar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+}
+__device__ __forceinline__ void brt_teardown(BrtSmem& S) {
+    tc_fence_before();
+    __syncthreads();
+    if (threadIdx.x < 32) tc_dealloc<512>(S.tmem);
+}
+
+// ---- the blind-rotation kernel: a1 linear combination, a2 mod switch, a3 ACC init, a4 630 CMux, a5 extract ---
+__global__ void __launch_bounds__(kTcThreads, 1) brt_kernel(BrArgs A, const uint32_t* __restrict__ bk4,
+                                                             const unsigned char* __restrict__ tcB,
+                                                             const uint2* __restrict__ tcTw) {
+    extern __shared__ __align__(1024) unsigned char brt_smem[];
+    BrtSmem& S = *reinterpret_cast<BrtSmem*>(brt_smem);
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int lane0 = blockIdx.x * kTcG;
+    brt_setup(S, tcB, tcTw);
+    // a1 + a2: 6 warps per lane
+    {
+        const int g = warp / 6, w6 = warp % 6;
+        const int gl = lane0 + g;
+        LaneDesc d = {0, -1, 0, 0, 0u, 0u, 0u, 0u};
+        if (gl < A.nlanes) d = A.lanes[gl];
+        const uint32_t* s0 = (d.sel & 3u) == 0 ? A.src0 : ((d.sel & 3u) == 1 ? A.src1 : A.src2);
+        const uint32_t sb = (d.sel >> 2) & 3u;
+        const uint32_t* s1 = sb == 0 ? A.src0 : (sb == 1 ? A.src1 : A.src2);
+        const uint32_t* pa = s0 + (int64_t)d.ia * A.src_stride;
+        const uint32_t* pb = d.ib >= 0 ? s1 + (int64_t)d.ib * A.src_stride : nullptr;
+        for (int w = w6 * 32 + lane; w <= kn; w += 192) {
+            uint32_t v = (gl < A.nlanes) ? (uint32_t)d.wa * __ldg(pa + w) : 0u;
+            if (pb) v += (uint32_t)d.wb * __ldg(pb + w);
+            if (w == kn) v += d.cst;
+            S.bar[g][w] = (uint16_t)((v + (1u << 20)) >> 21);      // round(v 2N / 2^32) mod 2N (C5)
+        }
+    }
+    __syncthreads();
+    // a3: ACC = (0, X^{-bbar} (mu, ..., mu))  (C6)
+    for (int k = tid; k < kTcG * kN; k += kTcThreads) {
+        const int gg = k / kN, c = k % kN;
+        const uint32_t bbar = S.bar[gg][kn];
+        S.acc[gg][0][c] = 0u;
+        S.acc[gg][1][c] = ((c + bbar) & (kTwoN - 1)) < (uint32_t)kN ? kMu : (uint32_t)(0u - kMu);
+    }
+    __syncthreads();
+    uint32_t phase = 0;
+    for (int i = 0; i < kn; i++) {
+        brt_digits(S, i);
+        brt_cmux_tail(S, bk4 + (size_t)i * kN * kBk4Rec, phase);
+    }
+    // a5: sample extraction, index 0 (C8)
+    for (int k = tid; k < kTcG * (kN + 1); k += kTcThreads) {
+        const int g = k / (kN + 1), j = k % (kN + 1);
+        const int gl = lane0 + g;
+        if (gl >= A.nlanes) continue;
+        uint32_t v;
+        if (j == 0) v = S.acc[g][0][0];
+        else if (j < kN) v = 0u - S.acc[g][0][kN - j];
+        else v = S.acc[g][1][0];
+        A.out[(int64_t)gl * A.out_stride + j] = v;
+    }
+    brt_teardown(S);
+}
+
+// ---- diagnostic: res[g][q] = sum_r d[g][r] (x) polys[r][q] mod 2^32 through one CMux tail (acc starts at 0) --
+__global__ void __launch_bounds__(kTcThreads, 1) brt_muladd_kernel(const int32_t* __restrict__ digits,
+                                                                    const uint32_t* __restrict__ bk4,
+                                                                    const unsigned char* __restrict__ tcB,
+                                                                    const uint2* __restrict__ tcTw,
+                                                                    uint32_t* __restrict__ res) {
+    extern __shared__ __align__(1024) unsigned char brt_smem[];
+    BrtSmem& S = *reinterpret_cast<BrtSmem*>(brt_smem);
+    const int tid = threadIdx.x;
+    brt_setup(S, tcB, tcTw);
+    for (int k = tid; k < kTcG * 2 * kN; k += kTcThreads) (&S.acc[0][0][0])[k] = 0u;
+    // digits [g][r][1024] -> A1 row (g*6 + r)*32 + k2, K byte k1
+    for (int e = tid; e < kTcPolys * kN; e += kTcThreads) {
+        const int P = e / kN, c = e % kN, k1 = c >> 5, k2 = c & 31;
+        S.A1[tc_off(P * 32 + k2, k1, kA1Lbo, kA1Sbo)] = (unsigned char)(digits[e] & 0xFF);
+    }
+    uint32_t phase = 0;
+    brt_cmux_tail(S, bk4, phase);
+    for (int k = tid; k < kTcG * 2 * kN; k += kTcThreads) res[k] = (&S.acc[0][0][0])[k];
+    brt_teardown(S);
+}
+
+// ---- load time: BK (torus, [n][6][2][N]) -> bk4[i][32 j1 + j2][r*6 + o], o = q*3 + m: the evaluation of part m
+// of BK_i[r][q] at psi^(2 j + 1), j = j1 + 32 j2, times N^-1 (Horner's rule; plain and exact, ~24 G mulmods)
+__global__ void __launch_bounds__(256) bk_to_bk4_kernel(const uint32_t* __restrict__ bk, uint32_t* __restrict__ bk4,
+                                                         const uint2* __restrict__ pts, uint32_t ninv,
+                                                         uint32_t ninvp, int npolys) {
+    __shared__ uint32_t x[kN];
+    const int task = blockIdx.x;                        // (i, r, q, m)
+    if (task >= npolys) return;
+    const int m = task % kParts, q = (task / kParts) % 2, r = (task / (2 * kParts)) % kRows, i = task / (2 * kParts * kRows);
+    const uint32_t* src = bk + (((size_t)i * kRows + r) * 2 + q) * kN;
+    for (int k = threadIdx.x; k < kN; k += blockDim.x) {
+        uint32_t v = src[k];
+        const int32_t p0 = ((int32_t)((v & 0x7FFu) << 21)) >> 21;
+        v = (v - (uint32_t)p0) >> 11;
+        const int32_t p1 = ((int32_t)((v & 0x7FFu) << 21)) >> 21;
+        v = (v - (uint32_t)p1) >> 11;
+        const int32_t p2 = ((int32_t)((v & 0x3FFu) << 22)) >> 22;
+        const int32_t pm = m == 0 ? p0 : (m == 1 ? p1 : p2);
+        x[k] = pm < 0 ? (uint32_t)(pm + (int32_t)kP) : (uint32_t)pm;
+    }
+    __syncthreads();
+    for (int j = threadIdx.x; j < kN; j += blockDim.x) {
+        const uint2 w = pts[j];                         // psi^(2 j + 1) and its Shoup companion
+        uint32_t acc = 0;
+        for (int k = kN - 1; k >= 0; k--) acc = red_2p(add_alu(shoup_mul(acc, w.x, w.y), x[k]));
+        acc = red_p(shoup_mul(acc, ninv, ninvp));
+        const int j1 = j & 31, j2 = j >> 5;
+        bk4[((size_t)i * kN + (j1 * 32 + j2)) * kBk4Rec + r * 6 + q * kParts + m] = acc;
+    }
+}
+
+static size_t brt_smem_bytes() { return sizeof(BrtSmem); }
+
+int launch_brt(const BrArgs& A, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw, cudaStream_t st) {
+    static_assert(sizeof(BrtSmem) <= 232448, "brt shared memory");
+    if (ensure_smem_attr<brt_kernel>(brt_smem_bytes())) return -1;
+    const int blocks = (A.nlanes + kTcG - 1) / kTcG;
+    if (blocks == 0) return 0;
+    brt_kernel<<<blocks, kTcThreads, brt_smem_bytes(), st>>>(A, bk4, tcB, tcTw);
+    return 0;
+}
+
+int launch_brt_muladd(const int32_t* digits, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw,
+                      uint32_t* res, cudaStream_t st) {
+    if (ensure_smem_attr<brt_muladd_kernel>(brt_smem_bytes())) return -1;
+    brt_muladd_kernel<<<1, kTcThreads, brt_smem_bytes(), st>>>(digits, bk4, tcB, tcTw, res);
+    return 0;
+}
+
+void launch_bk_to_bk4(const uint32_t* bk, uint32_t* bk4, const uint2* pts, uint32_t ninv, uint32_t ninvp, int n_i,
+                      cudaStream_t st) {
+    const int npolys = n_i * kRows * 2 * kParts;
+    bk_to_bk4_kernel<<<npolys, 256, 0, st>>>(bk, bk4, pts, ninv, ninvp, npolys);
+}
+
+size_t bk4_bytes() { return (size_t)kn * kN * kBk4Rec * 4; }
+
+// host: constant B operands and twiddle tables of the four-step transform for the root psi
+void brt_tables(uint32_t psi, unsigned char* B, uint2* tw, uint2* pts) {
+    auto powm = [](uint64_t b, uint64_t e) {
+        uint64_t r = 1;
+        b %= kP;
+        while (e) {
+            if (e & 1) r = r * b % kP;
+            b = b * b % kP;
+            e >>= 1;
+        }
+        return (uint32_t)r;
+    };
+    auto pw = [&](int64_t e) { return powm(psi, (uint64_t)(((e % 2048) + 2048) % 2048)); };
+    auto shoup = [](uint32_t w) { return (uint32_t)(((uint64_t)w << 32) / kP); };
+    auto byte = [](uint32_t v, int b) { return (unsigned char)((v >> (8 * b)) & 0xFFu); };
+    auto dense = [](uint32_t n, uint32_t k, uint32_t K) { return tc_off(n, k, 128, (K / 16) * 128); };
+    memset(B, 0, kTcBTotal);
+    for (int j1 = 0; j1 < 32; j1++)                       // B1[(j1, b)][k1] = byte_b(W1[j1][k1])
+        for (int k1 = 0; k1 < 32; k1++)
+            for (int b = 0; b < 4; b++) B[dense(4 * j1 + b, k1, 32)] = byte(pw(32 * (2 * j1 + 1) * k1), b);
+    unsigned char* B2 = B + kB1Bytes;
+    unsigned char* B3 = B2 + kBBytes;
+    unsigned char* B4 = B3 + kBBytes;
+    for (int x = 0; x < 32; x++)
+        for (int y = 0; y < 32; y++)
+            for (int c = 0; c < 4; c++) {
+                const uint64_t s = ((uint64_t)1 << (8 * c)) % kP;
+                // B2[(j2 = x, b)][(k2 = y, c)] = byte_b(2^(8c) W2[j2][k2]), W2 = psi^(64 j2 k2)
+                const uint32_t w2 = (uint32_t)(s * pw(64 * x * y) % kP);
+                // B3[(k2 = x, b)][(j2 = y, c)] = byte_b(2^(8c) V2[k2][j2]), V2 = psi^(-64 j2 k2)
+                const uint32_t v2 = (uint32_t)(s * pw(-64 * x * y) % kP);
+                // B4[(k1 = x, b)][(j1 = y, c)] = byte_b(2^(8c) V1[k1][j1]), V1 = psi^(-32 (2 j1 + 1) k1)
+                const uint32_t v1 = (uint32_t)(s * pw(-32 * (2 * y + 1) * x) % kP);
+                for (int b = 0; b < 4; b++) {
+                    B2[dense(4 * x + b, 4 * y + c, 128)] = byte(w2, b);
+                    B3[dense(4 * x + b, 4 * y + c, 128)] = byte(v2, b);
+                    B4[dense(4 * x + b, 4 * y + c, 128)] = byte(v1, b);
+                }
+            }
+    for (int j1 = 0; j1 < 32; j1++)
+        for (int k2 = 0; k2 < 32; k2++) {
+            const uint32_t f = pw((2 * j1 + 1) * k2), iv = pw(-(2 * j1 + 1) * k2);
+            tw[j1 * 32 + k2] = make_uint2(f, shoup(f));            // twF[j1][k2]
+            tw[1024 + k2 * 32 + j1] = make_uint2(iv, shoup(iv));    // twI[k2][j1]
+        }
+    for (int j = 0; j < kN; j++) {
+        const uint32_t w = pw(2 * j + 1);
+        pts[j] = make_uint2(w, shoup(w));
+    }
+}
+size_t brt_table_bytes() { return kTcBTotal; }
+
+}  // namespace tb

@@ -95,3 +95,15 @@ size_t bkf_bytes();
 int launch_brl(const BrArgs& A, const double2* bkf, const double2* twL, cudaStream_t st);
 int brl_wave_lanes();
 }  // namespace tb
+
+namespace tb {
+// tensor-core blind rotation (tb_brt.cu)
+int launch_brt(const BrArgs& A, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw, cudaStream_t st);
+int launch_brt_muladd(const int32_t* digits, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw,
+                      uint32_t* res, cudaStream_t st);
+void launch_bk_to_bk4(const uint32_t* bk, uint32_t* bk4, const uint2* pts, uint32_t ninv, uint32_t ninvp, int n_i,
+                      cudaStream_t st);
+size_t bk4_bytes();
+void brt_tables(uint32_t psi, unsigned char* B, uint2* tw, uint2* pts);
+size_t brt_table_bytes();
+}  // namespace tb

@@ -77,6 +77,10 @@ struct tb_ctx {
     double2* fftC = nullptr;
     double2* fftL = nullptr;                // brl: [64][6] per-thread pass-2/3 twiddle bases
     uint32_t ninv = 0, ninvp = 0;
+    unsigned char* tcB = nullptr;           // tensor-core NTT: constant B operands (tb_brt.cu)
+    uint2* tcTw = nullptr;                  // [2][32][32] four-step twiddles (+ Shoup)
+    uint2* tcPts = nullptr;                 // [N] psi^(2j+1) (+ Shoup): evaluation points of bk4
+    uint32_t* bk4 = nullptr;                // [n][N][36] NTT-domain BK in the four-step order (brt_kernel)
     uint32_t* bkhat = nullptr;              // [n][6][6][N]
     double2* bkf = nullptr;                 // FP64 variant: [n][6][4][512] complex, scaled by 1/512
     uint32_t* ksk = nullptr;                // [N][t][3][632]
@@ -242,6 +246,9 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
     }
     c->ninv = powmod(kN, kP - 2);
     c->ninvp = shoup_of(c->ninv);
+    std::vector<unsigned char> tcb(brt_table_bytes());
+    std::vector<uint2> tctw(2048), tcpts(kN);
+    brt_tables(psi, tcb.data(), tctw.data(), tcpts.data());
     int rc = set_ntt_constants(fw, fwp, iw, iwp, misc);
     if (rc == 0) rc = set_fft_constants(zeta16.data());
     cudaError_t e = cudaSuccess;
@@ -251,6 +258,12 @@ extern "C" int tb_ctx_create(const tb_params* P, int dev, tb_ctx** out) {
     if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->fftC, fc.data(), fc.size() * sizeof(double2), cudaMemcpyHostToDevice);
     if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->fftL, fl.size() * sizeof(double2));
     if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->fftL, fl.data(), fl.size() * sizeof(double2), cudaMemcpyHostToDevice);
+    if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->tcB, tcb.size());
+    if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->tcB, tcb.data(), tcb.size(), cudaMemcpyHostToDevice);
+    if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->tcTw, tctw.size() * sizeof(uint2));
+    if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->tcTw, tctw.data(), tctw.size() * sizeof(uint2), cudaMemcpyHostToDevice);
+    if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->tcPts, tcpts.size() * sizeof(uint2));
+    if (rc == 0 && e == cudaSuccess) e = cudaMemcpy(c->tcPts, tcpts.data(), tcpts.size() * sizeof(uint2), cudaMemcpyHostToDevice);
     if (rc == 0 && e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->own, cudaStreamNonBlocking);
     if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->twF, 31 * 32 * sizeof(uint2));
     if (rc == 0 && e == cudaSuccess) e = cudaMalloc(&c->twI, 31 * 32 * sizeof(uint2));
@@ -273,6 +286,10 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
     cudaFree(c->fftC);
     cudaFree(c->fftL);
     cudaFree(c->bkhat);
+    cudaFree(c->bk4);
+    cudaFree(c->tcB);
+    cudaFree(c->tcTw);
+    cudaFree(c->tcPts);
     cudaFree(c->bkf);
     cudaFree(c->ksk);
     cudaFree(c->lanebuf);
@@ -319,8 +336,8 @@ extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
 }
 
 extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
-    if (!c || !(variant == 6 || variant == 10))
-        return fail(TB_EINVAL, "blind-rotation variant must be 6 or 10");
+    if (!c || !(variant == 6 || variant == 10 || variant == 12))
+        return fail(TB_EINVAL, "blind-rotation variant must be 6, 10 or 12");
     c->variant = variant;
     return TB_OK;
 }
@@ -364,12 +381,14 @@ extern "C" int tb_load_bk(tb_ctx* c, const uint32_t* host_bk, size_t n_words) {
     TB_CUDA(cudaSetDevice(c->device));
     if (!c->bkhat) TB_CUDA(cudaMalloc(&c->bkhat, (size_t)kn * kRows * kOuts * kN * 4));
     if (!c->bkf) TB_CUDA(cudaMalloc(&c->bkf, bkf_bytes()));
+    if (!c->bk4) TB_CUDA(cudaMalloc(&c->bk4, bk4_bytes()));
     uint32_t* tmp = nullptr;
     TB_CUDA(cudaMalloc(&tmp, want * 4));
     cudaError_t e = cudaMemcpyAsync(tmp, host_bk, want * 4, cudaMemcpyHostToDevice, c->own);
     if (e == cudaSuccess) {
         launch_bk_to_ntt(tmp, c->bkhat, c->twF, c->ninv, c->ninvp, c->own);
         launch_bk_to_fft(tmp, c->bkf, c->fftB, c->fftC, c->own);
+        launch_bk_to_bk4(tmp, c->bk4, c->tcPts, c->ninv, c->ninvp, kn, c->own);
         e = cudaGetLastError();
     }
     if (e == cudaSuccess) e = cudaStreamSynchronize(c->own);
@@ -445,6 +464,8 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     if (c->narrow_lanes > 0 && nlanes <= c->narrow_lanes)
         rc = nk == 9 ? launch_br9(A, st)                       // narrow level: one lane per 2-SM cluster
                      : launch_brl(A, c->bkf, c->fftL, st);     // or per 4-SM cluster (FP64)
+    else if (c->variant == 12)
+        rc = launch_brt(A, c->bk4, c->tcB, c->tcTw, st);
     else if (c->variant == 10)
         rc = launch_brf(A, c->lanes_per_cta ? std::min(c->lanes_per_cta, 3) : 2, c->bkf, c->fftB, c->fftC, st);
     else
@@ -603,6 +624,20 @@ extern "C" int tb_microbench_fields(tb_ctx* c, int iters, double* rates) {
     if (!c || !rates || iters <= 0) return fail(TB_EINVAL, "bad argument");
     TB_CUDA(cudaSetDevice(c->device));
     if (run_microbench_fields(iters, rates)) return fail(TB_ECUDA, "microbenchmark failed");
+    return TB_OK;
+}
+
+extern "C" int tb_tc_muladd(tb_ctx* c, const int32_t* digits, const uint32_t* polys, uint32_t* res) {
+    if (!c || !digits || !polys || !res) return fail(TB_EINVAL, "null argument");
+    TB_CUDA(cudaSetDevice(c->device));
+    uint32_t* b4 = nullptr;
+    TB_CUDA(cudaMalloc(&b4, (size_t)kN * 36 * 4));
+    launch_bk_to_bk4(polys, b4, c->tcPts, c->ninv, c->ninvp, 1, c->own);
+    const int rc = launch_brt_muladd(digits, b4, c->tcB, c->tcTw, res, c->own);
+    cudaError_t e = rc ? cudaErrorLaunchFailure : cudaGetLastError();
+    if (e == cudaSuccess) e = cudaStreamSynchronize(c->own);
+    cudaFree(b4);
+    if (e != cudaSuccess) return cuda_fail(e, "tb_tc_muladd");
     return TB_OK;
 }
 

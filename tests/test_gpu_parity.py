@@ -113,9 +113,10 @@ def test_narrow_level_latency_mode_bit_exact(tb, ctx, keys, kernel):
         ctx.set_narrow_kernel(0)
 
 
-@pytest.mark.parametrize("variant", [6, 10])
+@pytest.mark.parametrize("variant", [6, 10, 12])
 def test_blind_rotation_variants_bit_exact(tb, ctx, keys, variant):
-    """every blind-rotation kernel variant (br6 integer NTT / brf FP64 FFT) on a ragged batch of 9"""
+    """every blind-rotation kernel variant (br6 integer NTT / brf FP64 FFT / brt tensor-core NTT) on a ragged
+    batch of 9"""
     rng = np.random.default_rng(40 + variant)
     cts = rng.integers(0, M32, (9, 631), dtype=np.uint64).astype(np.uint32)
     ctx.set_br_variant(variant)
@@ -375,7 +376,7 @@ def test_mixed_netlist_with_not_and_mux(tb, ctx, keys):
     assert (O.decrypt_bits(keys, gpu) == plain).all()
 
 
-@pytest.mark.parametrize("variant", [6, 10])
+@pytest.mark.parametrize("variant", [6, 10, 12])
 def test_throughput_level_bench_size_sampled(tb, ctx, keys, variant):
     """BASELINE configs[2] at the bench's per-GPU size (65,536 NAND/XOR gates, one level, the launch
     configuration bench.py times, default br6 and --br-variant 10): all outputs decrypt to the truth; a
