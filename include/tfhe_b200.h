@@ -220,7 +220,7 @@ int tb_microbench(tb_ctx* ctx, int iters, double* butterflies_per_s, double* mac
  * own), Goldilocks general-twiddle butterflies/s, Goldilocks shift-twiddle (x 2^s) butterflies/s, 64-bit
  * MACs/s.  Synchronous; iters <= 0 or null pointers: TB_EINVAL. */
 int tb_microbench_fields(tb_ctx* ctx, int iters, double* rates);
-/* Tensor-core external-product core (diagnostic): for two lanes g and both output polynomials q,
+/* Tensor-core external-product core (diagnostic): for four lanes g and both output polynomials q,
  * res[g][q][.] = sum_{r<6} digits[g][r] (x) polys[r][q] mod 2^32 (negacyclic), computed exactly as one CMux step
  * of the tensor-core blind rotation does it (four-step NTT on tcgen05 kind::i8, MAC against the NTT-domain BK,
  * inverse, centred lift).  Device pointers: digits int32 [2][6][1024] in [-64, 63],

@@ -230,8 +230,8 @@ class Context:
                 "mac64_per_s": r[3]}
 
     def tc_muladd(self, digits: torch.Tensor, polys: torch.Tensor) -> torch.Tensor:
-        """diagnostic: [2][2][1024] = sum_r digits[g][r] (x) polys[r][q] through the tensor-core CMux (tb_tc_muladd)"""
-        res = torch.empty((2, 2, N_RING), dtype=torch.int32, device=self.device)
+        """diagnostic: [4][2][1024] = sum_r digits[g][r] (x) polys[r][q] through the tensor-core CMux (tb_tc_muladd)"""
+        res = torch.empty((4, 2, N_RING), dtype=torch.int32, device=self.device)
         d, p = digits.contiguous(), polys.contiguous()
         _native.check(_native.lib().tb_tc_muladd(self._h, _ptr(d), _ptr(p), _ptr(res)))
         return res

@@ -20,8 +20,15 @@
 // u8 x u8 (digits: s8 x u8) with K = 32 (digits) or 128 and N = 128 (4 limbs x 32), and the CUDA cores only
 // recombine the 4 limbs (one Shoup product by 2^16) and apply the twiddles.
 //
-// A CTA = G = 2 lanes (bootstraps) = 12 polynomials per transform = three M = 128 tiles; one CTA per SM;
-// accumulators resident in shared memory for all n = 630 CMux steps; 12 warps, thread 0 issues the MMAs.
+// Structure (one CTA per SM, G = 4 lanes = bootstraps, accumulators resident in shared memory for all n = 630
+// CMux steps).  A CMux step is 4 GEMM stages x 6 tile jobs (a tile = 4 polynomials = 128 rows):
+//   digits (all compute warps) -> GEMM1 -> ep1 (limbs, twiddle) -> GEMM2 -> ep2 (limbs) -> MAC (all compute
+//   warps; each NTT-domain BK word read once for the 4 lanes) -> GEMM3 -> ep3 (limbs, twiddle) -> GEMM4 -> ep4
+//   (limbs, lift, ACC +=).
+// Warp 12 issues the MMAs (one thread) into a ring of 4 TMEM slots (128 columns each) and runs ahead of the 12
+// compute warps (3 quads of 4 warps, one warp per TMEM lane quadrant); a quad takes every third tile job of a
+// stage.  mbarriers: full[slot] (MMA commit -> epilogue), empty[slot] (4 epilogue warps -> MMA), a2[tile] (ep1
+// wrote GEMM2's operand tile), gate (all 12 compute warps done with digits / MAC / ep3).
 #include <cstring>
 
 #include "tb_kernels.cuh"
@@ -30,13 +37,16 @@
 
 namespace tb {
 
-constexpr int kTcG = 2;                       // lanes per CTA
-constexpr int kTcPolys = 6 * kTcG;            // polynomials per transform stage (12 = 3 tiles of 4)
-constexpr int kTcWarps = 12;
-constexpr int kTcThreads = 32 * kTcWarps;
+constexpr int kTcG = 4;                       // lanes per CTA
+constexpr int kTcPolys = 6 * kTcG;            // polynomials per transform stage (24 = 6 tiles of 4)
+constexpr int kTcTiles = kTcPolys / 4;
+constexpr int kTcCompWarps = 12;
+constexpr int kTcCompThreads = 32 * kTcCompWarps;
+constexpr int kTcThreads = kTcCompThreads + 32;         // + the MMA warp
+constexpr int kTcSlots = 4;                              // TMEM ring: 4 x 128 columns
 // shared-memory operand layouts (K-major core matrices, tb_tc.cuh)
-constexpr uint32_t kA1Lbo = 128, kA1Sbo = 256;          // digits: 384 rows x 32 B
-constexpr uint32_t kOpLbo = 144, kOpSbo = 8 * 144;      // 30-bit operands: 3 tiles x 128 rows x 128 B (padded)
+constexpr uint32_t kA1Lbo = 128, kA1Sbo = 256;          // digits: 128 rows x 32 B per tile (at the tile's start)
+constexpr uint32_t kOpLbo = 144, kOpSbo = 8 * 144;      // 30-bit operands: 128 rows x 128 B per tile (padded)
 constexpr uint32_t kOpTile = 16 * kOpSbo;               // 18,432 B
 constexpr uint32_t kB1Bytes = 128 * 32, kBBytes = 128 * 128;
 constexpr uint32_t kTcBTotal = kB1Bytes + 3 * kBBytes;  // B1 (W1 bytes), B2 (W2'), B3 (V2'), B4 (V1')
@@ -44,249 +54,264 @@ constexpr int kBk4Rec = 36;                              // NTT-domain BK record
 
 struct BrtSmem {
     unsigned char B[kTcBTotal];                  // constant B operands (dense: LBO 128)
-    unsigned char A1[kTcPolys * 32 * 32];        // digit operand
-    unsigned char op[3 * kOpTile];               // 30-bit operand / MAC buffer (A2, MAC in/out = A3, A4)
+    unsigned char op[kTcTiles * kOpTile];        // per tile: A1 | A2 | MAC in / out = A3 | A4 (stage-aliased)
     uint2 twF[32 * 32];                          // [j1][k2] (psi^((2 j1 + 1) k2), Shoup)
     uint2 twI[32 * 32];                          // [k2][j1] (psi^(-(2 j1 + 1) k2), Shoup)
     uint32_t acc[kTcG][2][kN];
     uint16_t bar[kTcG][kn + 2];
-    uint64_t mbar;
+    uint64_t full[kTcSlots], empty[kTcSlots], a2[kTcTiles], gate;
     uint32_t tmem;
 };
 
-// ---- limb recombination: sum_b 2^(8 b) Y_b mod p, result in [0, 4p) --------------------------------
-constexpr uint32_t kW16 = 1u << 16;
+// ---- limb recombination: sum_b 2^(8 b) Y_b mod p ----------------------------------------------------------
 constexpr uint32_t kW16p = (uint32_t)((((uint64_t)1 << 48)) / kP);    // Shoup companion of 2^16
+// operands < 2p (top byte <= 127): Y0 + 2^8 Y1 <= 32 (3*255 + 127) 255 * 257 < 1.9e9, hi 2^16 mod p < 2p,
+// so the sum stays below 4.1e9 < 4p: no reduction of the low half is needed
 __device__ __forceinline__ uint32_t limbs_u(uint32_t y0, uint32_t y1, uint32_t y2, uint32_t y3) {
-    const uint32_t lo = y0 + (y1 << 8), hi = y2 + (y3 << 8);           // each < 2^31 + 2^23 < 4p
+    const uint32_t lo = y0 + (y1 << 8), hi = y2 + (y3 << 8);
     const uint32_t q = __umulhi(hi, kW16p);
-    const uint32_t r = (hi << 16) - q * kP;                            // hi 2^16 mod p in [0, 2p)
-    return red_2p(lo) + r;
+    return lo + ((hi << 16) - q * kP);
 }
+// signed limbs (s8 digits x u8, |Y_b| < 2^19): lo + p, hi + p are in (0, 2p); result < 4p
 __device__ __forceinline__ uint32_t limbs_s(uint32_t y0, uint32_t y1, uint32_t y2, uint32_t y3) {
-    // signed limbs (s8 digits x u8): |Y_b| < 2^19, so lo + p, hi + p are in (0, 2p)
     const uint32_t lo = y0 + (y1 << 8) + kP, hi = y2 + (y3 << 8) + kP;
     const uint32_t q = __umulhi(hi, kW16p);
-    const uint32_t r = (hi << 16) - q * kP;
-    return lo + r;
+    return lo + ((hi << 16) - q * kP);
 }
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void comp_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kTcCompThreads) : "memory"); }
 
-// ---- one GEMM stage: tiles x K-steps, one commit ------------------------------------------------------
-__device__ __forceinline__ void brt_gemm(const BrtSmem& S, uint32_t tmem, int stage) {
-    // stage 0: A1 x B1 (K = 32, s8 digits); 1: op x B2; 2: op x B3; 3: op (tile m) x B4 -> columns 128 m
-    const uint32_t sB = smem_u32(S.B), sA1 = smem_u32(S.A1), sOp = smem_u32(S.op);
-    if (stage == 0) {
-        constexpr uint32_t id = tc_idesc_i8(128, 128, true, false);
-        for (int t = 0; t < 3; t++)
-            tc_mma_i8(tmem + 128 * t, tc_sdesc(sA1 + t * 16 * kA1Sbo, kA1Lbo, kA1Sbo), tc_sdesc(sB, 128, 256), id, 0);
-    } else {
-        constexpr uint32_t id = tc_idesc_i8(128, 128, false, false);
-        const uint32_t bb = sB + kB1Bytes + (stage - 1) * kBBytes;
-        for (int t = 0; t < 3; t++)
-            for (int s = 0; s < 4; s++)
-                tc_mma_i8(tmem + 128 * t, tc_sdesc(sOp + t * kOpTile + 2 * s * kOpLbo, kOpLbo, kOpSbo),
-                          tc_sdesc(bb + 2 * s * 128, 128, 1024), id, s > 0);
+// byte offset of (row, 32-bit word) of an operand tile
+__host__ __device__ constexpr uint32_t opw(uint32_t row, uint32_t word) { return tc_off(row, 4 * word, kOpLbo, kOpSbo); }
+
+// ---- MMA warp: the static job sequence of one CMux step (stage s, tile t), job counter k across steps -------
+__device__ __forceinline__ void brt_mma_step(BrtSmem& S, uint32_t& k, uint32_t& gate_ph, uint32_t& a2_ph) {
+    const uint32_t sB = smem_u32(S.B), sOp = smem_u32(S.op);
+    constexpr uint32_t id_s = tc_idesc_i8(128, 128, true, false), id_u = tc_idesc_i8(128, 128, false, false);
+    for (int s = 0; s < 4; s++) {
+        if (s != 1) {                                   // digits / MAC / ep3 of every compute warp done
+            mbar_wait(&S.gate, gate_ph);
+            gate_ph ^= 1;
+        }
+        for (int t = 0; t < kTcTiles; t++, k++) {
+            const uint32_t slot = k % kTcSlots;
+            if (s == 1) mbar_wait(&S.a2[t], a2_ph);     // ep1 wrote this tile's GEMM2 operand
+            if (k >= kTcSlots) mbar_wait(&S.empty[slot], ((k / kTcSlots) - 1) & 1);
+            tc_fence_after();
+            const uint32_t d = S.tmem + 128 * slot;
+            const uint32_t a = sOp + t * kOpTile;
+            if (s == 0) {
+                tc_mma_i8(d, tc_sdesc(a, kA1Lbo, kA1Sbo), tc_sdesc(sB, 128, 256), id_s, 0);
+            } else {
+                const uint32_t bb = sB + kB1Bytes + (s - 1) * kBBytes;
+#pragma unroll
+                for (int q = 0; q < 4; q++)
+                    tc_mma_i8(d, tc_sdesc(a + 2 * q * kOpLbo, kOpLbo, kOpSbo), tc_sdesc(bb + 2 * q * 128, 128, 1024),
+                              id_u, q > 0);
+            }
+            tc_commit(smem_u32(&S.full[slot]));
+        }
+        if (s == 1) a2_ph ^= 1;
     }
-    tc_commit(smem_u32(&S.mbar));
 }
 
-__device__ __forceinline__ uint32_t op_word_off(int row, int word) { return tc_off(row, 4 * word, kOpLbo, kOpSbo); }
+// ---- compute warps ---------------------------------------------------------------------------------------
+// digits of (X^abar - 1) ACC for the 4 lanes -> A1 (a4.1).  Task (g, bloc, k2, h): coefficients
+// c = 32 (16 h + u) + k2, u < 16; digit jd of polynomial P = g*6 + bloc*3 + jd goes to tile P / 4, row
+// (P % 4)*32 + k2, K bytes 16 h .. 16 h + 15 (one 16-byte store)
+__device__ __forceinline__ void brt_digits(BrtSmem& S, int i) {
+    for (int task = threadIdx.x; task < kTcG * 2 * 32 * 2; task += kTcCompThreads) {
+        const int k2 = task & 31, h = (task >> 5) & 1, bloc = (task >> 6) & 1, g = task >> 7;
+        const uint32_t ab = S.bar[g][i];
+        const uint32_t* acc = S.acc[g][bloc];
+        uint32_t d[3][4] = {};
+#pragma unroll
+        for (int u = 0; u < 16; u++) {
+            const uint32_t c = 32u * (16 * h + u) + k2;
+            const uint32_t mm = (c - ab) & (kTwoN - 1);
+            const uint32_t src = acc[mm & (kN - 1)];
+            const uint32_t rot = mm < (uint32_t)kN ? src : 0u - src;
+            const uint32_t x = rot - acc[c] + c_misc[3];             // (X^abar - 1) ACC + decomposition offset
+#pragma unroll
+            for (int jd = 0; jd < 3; jd++) {
+                const uint32_t dig = ((x >> (32 - kBgbit * (jd + 1))) & 127u) - 64u;   // digit in [-64, 63]
+                d[jd][u >> 2] |= (dig & 0xFFu) << (8 * (u & 3));
+            }
+        }
+#pragma unroll
+        for (int jd = 0; jd < 3; jd++) {
+            const int P = g * 6 + bloc * 3 + jd;
+            *reinterpret_cast<uint4*>(S.op + (P >> 2) * kOpTile + tc_off((P & 3) * 32 + k2, 16 * h, kA1Lbo, kA1Sbo)) =
+                make_uint4(d[jd][0], d[jd][1], d[jd][2], d[jd][3]);
+        }
+    }
+}
 
-// ---- the CMux pipeline after the digits are in A1 (shared by the kernel and the diagnostic) ----------
-// bk4: this step's NTT-domain BK records [32 j1 + j2][36]; out: ep4 result added into acc[g][q][.]
-__device__ __forceinline__ void brt_cmux_tail(BrtSmem& S, const uint32_t* __restrict__ bk4, uint32_t& phase) {
+// Where the MAC writes output o of lane g (and so where GEMM3 / ep3 / GEMM4 / ep4 find it): tile
+// (m = o % 3) * 2 + g / 2, quadrant (g % 2) * 2 + q (q = o / 3).  Then GEMM3's tile (m, h) holds exactly the
+// polynomials whose ep3 output fills A4 tile (m, h): ep3 rewrites only the tile it has just consumed.
+__device__ __forceinline__ int mac_out_tile(int g, int o) { return (o % 3) * 2 + (g >> 1); }
+__device__ __forceinline__ int mac_out_quad(int g, int o) { return (g & 1) * 2 + o / 3; }
+
+// The compute warps' part of one CMux step; k = job counter (same sequence as the MMA warp)
+__device__ __forceinline__ void brt_comp_step(BrtSmem& S, const uint32_t* __restrict__ bk4, uint32_t& k,
+                                              uint32_t* __restrict__ res_debug = nullptr) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint32_t tq = S.tmem + ((uint32_t)(32 * (warp & 3)) << 16);   // this warp's TMEM lane quadrant
-    const int t = warp >> 2;                                           // tile of polynomial P = warp
-    const int P = warp;
-    // GEMM1: digits x W1
+    const int quad = warp >> 2, qd = warp & 3;
+    const uint32_t tq = S.tmem + ((uint32_t)(32 * qd) << 16);     // this warp's TMEM lane quadrant
+    // digits were written by the caller; publish them to the MMA warp
     fence_async_smem();
-    tc_fence_before();
-    __syncthreads();
-    if (tid == 0) {
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.gate);
+    // ---- ep1: job (0, t), t % 3 == quad: thread (P = 4t + qd, k2 = lane): C[j1][k2] -> A2 row (qd, j1) word k2
+    for (int t = quad; t < kTcTiles; t += 3) {
+        const uint32_t kk = k + t, slot = kk % kTcSlots;
+        mbar_wait(&S.full[slot], (kk / kTcSlots) & 1);
         tc_fence_after();
-        brt_gemm(S, S.tmem, 0);
-    }
-    mbar_wait(&S.mbar, phase);
-    phase ^= 1;
-    tc_fence_after();
-    // ep1: thread (P, k2 = lane): B[j1][k2] -> C = B . psi^((2 j1 + 1) k2) -> op row (P, j1), word k2
-    {
-        const int k2 = lane;
+        unsigned char* base = S.op + t * kOpTile + opw(qd * 32, lane);
+        const uint2* tw = S.twF + lane;
+#pragma unroll
         for (int jc = 0; jc < 8; jc++) {
             uint32_t v[16];
-            tc_ld16(tq + 128 * t + 16 * jc, v);
+            tc_ld16(tq + 128 * slot + 16 * jc, v);
             tc_wait_ld();
 #pragma unroll
             for (int u = 0; u < 4; u++) {
                 const int j1 = 4 * jc + u;
                 const uint32_t x = limbs_s(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3]);
-                const uint2 w = S.twF[j1 * 32 + k2];
-                *reinterpret_cast<uint32_t*>(S.op + t * kOpTile + op_word_off((P & 3) * 32 + j1, k2)) =
-                    shoup_mul(x, w.x, w.y);
+                const uint2 w = tw[32 * j1];
+                *reinterpret_cast<uint32_t*>(base + (j1 >> 3) * kOpSbo + (j1 & 7) * 16) = shoup_mul(x, w.x, w.y);
             }
         }
+        fence_async_smem();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+            mbar_arrive(&S.empty[slot]);
+            mbar_arrive(&S.a2[t]);
+        }
     }
-    fence_async_smem();
-    tc_fence_before();
-    __syncthreads();
-    if (tid == 0) {
+    k += kTcTiles;
+    // ---- ep2: job (1, t): thread (P = 4t + qd, j1 = lane): A[j1 + 32 j2] in [0, 2p) -> row (qd, j1) words j2
+    for (int t = quad; t < kTcTiles; t += 3) {
+        const uint32_t kk = k + t, slot = kk % kTcSlots;
+        mbar_wait(&S.full[slot], (kk / kTcSlots) & 1);
         tc_fence_after();
-        brt_gemm(S, S.tmem, 1);
-    }
-    mbar_wait(&S.mbar, phase);
-    phase ^= 1;
-    tc_fence_after();
-    // ep2: thread (P, j1 = lane): A[j1 + 32 j2] for j2 = 4c..4c+3 -> [0, 2p) -> op row (P, j1), words 4c..4c+3
-    {
-        const int j1 = lane;
-        unsigned char* rowp = S.op + t * kOpTile;
+        unsigned char* base = S.op + t * kOpTile + opw(qd * 32 + lane, 0);
+#pragma unroll
         for (int c = 0; c < 8; c++) {
             uint32_t v[16];
-            tc_ld16(tq + 128 * t + 16 * c, v);
+            tc_ld16(tq + 128 * slot + 16 * c, v);
             tc_wait_ld();
             uint4 o;
             o.x = red_2p(limbs_u(v[0], v[1], v[2], v[3]));
             o.y = red_2p(limbs_u(v[4], v[5], v[6], v[7]));
             o.z = red_2p(limbs_u(v[8], v[9], v[10], v[11]));
             o.w = red_2p(limbs_u(v[12], v[13], v[14], v[15]));
-            *reinterpret_cast<uint4*>(rowp + op_word_off((P & 3) * 32 + j1, 4 * c)) = o;
+            *reinterpret_cast<uint4*>(base + c * kOpLbo) = o;
         }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&S.empty[slot]);
     }
-    tc_fence_before();
-    __syncthreads();
-    // MAC: coefficient (j1, j2) of both lanes: M_o = sum_r A_r . BK4[r][o] (a4.3), in place (o reuses row r = o)
+    k += kTcTiles;
+    comp_sync();                                    // every ep2 tile written
+    // ---- MAC: coefficient (j1, j2) of the 4 lanes, M_o = sum_r A_r BK4[r][o] (a4.3); each BK word read once
     {
         const uint32_t R = c_misc[0], Rp = c_misc[1];
-        for (int pos = tid; pos < kN; pos += kTcThreads) {
-            const int j1 = pos >> 5, j2 = pos & 31;
+        const uint32_t lanew = (lane >> 2) * kOpLbo + (lane & 3) * 4;     // word j2 = lane within a row
+        for (int j1 = warp; j1 < 32; j1 += kTcCompWarps) {
+            const int pos = j1 * 32 + lane;
             const uint4* rec = reinterpret_cast<const uint4*>(bk4 + (size_t)pos * kBk4Rec);
             uint32_t B[kBk4Rec];
 #pragma unroll
-            for (int k = 0; k < kBk4Rec / 4; k++) {
-                const uint4 b4 = __ldg(rec + k);
-                B[4 * k] = b4.x; B[4 * k + 1] = b4.y; B[4 * k + 2] = b4.z; B[4 * k + 3] = b4.w;
+            for (int q = 0; q < kBk4Rec / 4; q++) {
+                const uint4 b4 = __ldg(rec + q);
+                B[4 * q] = b4.x; B[4 * q + 1] = b4.y; B[4 * q + 2] = b4.z; B[4 * q + 3] = b4.w;
             }
+            const uint32_t rowoff = (j1 >> 3) * kOpSbo + (j1 & 7) * 16 + lanew;
+            uint32_t D[kTcG][6];
 #pragma unroll
-            for (int g = 0; g < kTcG; g++) {
-                uint32_t* w[6];
-                uint32_t D[6];
+            for (int g = 0; g < kTcG; g++)
 #pragma unroll
                 for (int r = 0; r < 6; r++) {
-                    const int PP = g * 6 + r;
-                    w[r] = reinterpret_cast<uint32_t*>(S.op + (PP >> 2) * kOpTile + op_word_off((PP & 3) * 32 + j1, j2));
-                    D[r] = *w[r];
+                    const int P = g * 6 + r;
+                    D[g][r] = *reinterpret_cast<const uint32_t*>(S.op + (P >> 2) * kOpTile + (P & 3) * 4 * kOpSbo + rowoff);
                 }
+#pragma unroll
+            for (int g = 0; g < kTcG; g++)
 #pragma unroll
                 for (int o = 0; o < 6; o++) {
                     uint64_t s = 0;
 #pragma unroll
-                    for (int r = 0; r < 6; r++) s += (uint64_t)D[r] * B[r * 6 + o];
+                    for (int r = 0; r < 6; r++) s += (uint64_t)D[g][r] * B[r * 6 + o];
                     const uint32_t hi = (uint32_t)(s >> 32), lo = (uint32_t)s;
-                    *w[o] = red_2p(shoup_mul(hi, R, Rp) + (lo - (lo >> 30) * kP));
+                    *reinterpret_cast<uint32_t*>(S.op + mac_out_tile(g, o) * kOpTile + mac_out_quad(g, o) * 4 * kOpSbo +
+                                                 rowoff) = red_2p(shoup_mul(hi, R, Rp) + (lo - (lo >> 30) * kP));
                 }
-            }
         }
     }
-    fence_async_smem();
-    tc_fence_before();
-    __syncthreads();
-    if (tid == 0) {
+    fence_async_smem();                             // (the MAC is in place per thread: one thread owns (j1, j2))
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.gate);
+    // ---- ep3: job (2, t = m*2 + h): thread (quadrant qd = (g%2)*2 + q, j1 = lane): D[j1][k2] -> E -> A4 tile t
+    // row (qd, k2) word j1 (the tile GEMM3 just consumed)
+    for (int t = quad; t < kTcTiles; t += 3) {
+        const uint32_t kk = k + t, slot = kk % kTcSlots;
+        mbar_wait(&S.full[slot], (kk / kTcSlots) & 1);
         tc_fence_after();
-        brt_gemm(S, S.tmem, 2);
-    }
-    mbar_wait(&S.mbar, phase);
-    phase ^= 1;
-    tc_fence_after();
-    // ep3: thread (O = g*6 + o, j1 = lane): D[j1][k2] -> E = D . psi^(-(2 j1 + 1) k2) -> A4 tile m = o % 3,
-    // row (g*2 + q)*32 + k2, word j1
-    {
-        const int j1 = lane, O = P, g = O / 6, o = O % 6, q = o / 3, m = o % 3;
-        unsigned char* dst = S.op + m * kOpTile;   // GEMM3 has consumed op (A3): it is rewritten as A4
+        unsigned char* base = S.op + t * kOpTile + opw(qd * 32, lane);
+        const uint2* tw = S.twI + lane;
+#pragma unroll
         for (int c = 0; c < 8; c++) {
             uint32_t v[16];
-            tc_ld16(tq + 128 * t + 16 * c, v);
+            tc_ld16(tq + 128 * slot + 16 * c, v);
             tc_wait_ld();
 #pragma unroll
             for (int u = 0; u < 4; u++) {
                 const int k2 = 4 * c + u;
                 const uint32_t x = limbs_u(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3]);
-                const uint2 w = S.twI[k2 * 32 + j1];
-                *reinterpret_cast<uint32_t*>(dst + op_word_off((g * 2 + q) * 32 + k2, j1)) = shoup_mul(x, w.x, w.y);
+                const uint2 w = tw[32 * k2];
+                *reinterpret_cast<uint32_t*>(base + (k2 >> 3) * kOpSbo + (k2 & 7) * 16) = shoup_mul(x, w.x, w.y);
             }
         }
+        fence_async_smem();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&S.empty[slot]);
     }
-    fence_async_smem();
-    tc_fence_before();
-    __syncthreads();
-    if (tid == 0) {
+    k += kTcTiles;
+    // GEMM4 needs every A4 tile: ep3 of every quad done
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&S.gate);
+    // ---- ep4: job (3, t = m*2 + h): thread (g = 2h + qd/2, q = qd%2, k2 = lane): part m of N a[32 k1 + k2] ->
+    // centred lift, << 11 m, added into ACC[g][q] (a4.4; the three part jobs of (g, q) add atomically)
+    for (int t = quad; t < kTcTiles; t += 3) {
+        const uint32_t kk = k + t, slot = kk % kTcSlots;
+        mbar_wait(&S.full[slot], (kk / kTcSlots) & 1);
         tc_fence_after();
-        const uint32_t sB4 = smem_u32(S.B) + kB1Bytes + 2 * kBBytes, sOp = smem_u32(S.op);
-        constexpr uint32_t id = tc_idesc_i8(128, 128, false, false);
-        for (int m = 0; m < 3; m++)
-            for (int s = 0; s < 4; s++)
-                tc_mma_i8(S.tmem + 128 * m, tc_sdesc(sOp + m * kOpTile + 2 * s * kOpLbo, kOpLbo, kOpSbo),
-                          tc_sdesc(sB4 + 2 * s * 128, 128, 1024), id, s > 0);
-        tc_commit(smem_u32(&S.mbar));
-    }
-    mbar_wait(&S.mbar, phase);
-    phase ^= 1;
-    tc_fence_after();
-    // ep4: thread (g, q, k2 = lane) [quadrant = g*2 + q]: the 3 parts of coefficient 32 k1 + k2 -> centred lift,
-    // << 11 m, summed into ACC (a4.4); the three warps of a quadrant split k1 in groups of 4
-    {
-        const int quad = warp & 3, g = quad >> 1, q = quad & 1, k2 = lane;
-        const int kg0 = (warp >> 2) * 3, kg1 = kg0 + 3 < 8 ? kg0 + 3 : 8;
-        for (int kg = kg0; kg < kg1; kg++) {
-            uint32_t v0[16], v1[16], v2[16];
-            tc_ld16(tq + 0 * 128 + 16 * kg, v0);
-            tc_ld16(tq + 1 * 128 + 16 * kg, v1);
-            tc_ld16(tq + 2 * 128 + 16 * kg, v2);
+        const int m = t >> 1, g = 2 * (t & 1) + (qd >> 1), q = qd & 1;
+        uint32_t* acc = &S.acc[g][q][lane];
+#pragma unroll
+        for (int c = 0; c < 8; c++) {
+            uint32_t v[16];
+            tc_ld16(tq + 128 * slot + 16 * c, v);
             tc_wait_ld();
 #pragma unroll
             for (int u = 0; u < 4; u++) {
-                const int k1 = 4 * kg + u;
-                const uint32_t a0 = lift_centred(red_2p(limbs_u(v0[4 * u], v0[4 * u + 1], v0[4 * u + 2], v0[4 * u + 3])));
-                const uint32_t a1 = lift_centred(red_2p(limbs_u(v1[4 * u], v1[4 * u + 1], v1[4 * u + 2], v1[4 * u + 3])));
-                const uint32_t a2 = lift_centred(red_2p(limbs_u(v2[4 * u], v2[4 * u + 1], v2[4 * u + 2], v2[4 * u + 3])));
-                uint32_t* acc = &S.acc[g][q][32 * k1 + k2];
-                *acc = *acc + a0 + (a1 << 11) + (a2 << 22);
+                const int k1 = 4 * c + u;
+                const uint32_t a = lift_centred(red_2p(limbs_u(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3])));
+                atomicAdd(acc + 32 * k1, a << (11 * m));
             }
         }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&S.empty[slot]);
     }
-    tc_fence_before();
-    __syncthreads();
-}
-
-// ---- digits of (X^abar - 1) ACC for both lanes -> A1 (a4.1) -----------------------------------------
-// task (g, bloc, k2, h): 16 coefficients c = 32 (16 h + i) + k2, three digit bytes each, one 16-B store per digit
-__device__ __forceinline__ void brt_digits(BrtSmem& S, int i) {
-    const int tid = threadIdx.x;
-    if (tid >= kTcG * 2 * 32 * 2) return;
-    const int k2 = tid & 31, h = (tid >> 5) & 1, bloc = (tid >> 6) & 1, g = tid >> 7;
-    const uint32_t ab = S.bar[g][i];
-    const uint32_t* acc = S.acc[g][bloc];
-    uint32_t d[3][4] = {};
-#pragma unroll
-    for (int u = 0; u < 16; u++) {
-        const uint32_t c = 32u * (16 * h + u) + k2;
-        const uint32_t mm = (c - ab) & (kTwoN - 1);
-        const uint32_t src = acc[mm & (kN - 1)];
-        const uint32_t rot = mm < (uint32_t)kN ? src : 0u - src;
-        const uint32_t x = rot - acc[c] + c_misc[3];             // (X^abar - 1) ACC + decomposition offset
-#pragma unroll
-        for (int jd = 0; jd < 3; jd++) {
-            const uint32_t dig = ((x >> (32 - kBgbit * (jd + 1))) & 127u) - 64u;   // digit in [-64, 63]
-            d[jd][u >> 2] |= (dig & 0xFFu) << (8 * (u & 3));
-        }
-    }
-#pragma unroll
-    for (int jd = 0; jd < 3; jd++) {
-        const int P = g * 6 + bloc * 3 + jd;
-        const uint32_t row = P * 32 + k2;
-        *reinterpret_cast<uint4*>(S.A1 + tc_off(row, 16 * h, kA1Lbo, kA1Sbo)) =
-            make_uint4(d[jd][0], d[jd][1], d[jd][2], d[jd][3]);
-    }
+    k += kTcTiles;
+    comp_sync();                                    // ACC complete before the next step's digits
 }
 
 __device__ __forceinline__ void brt_setup(BrtSmem& S, const unsigned char* tcB, const uint2* tcTw) {
@@ -297,9 +322,14 @@ __device__ __forceinline__ void brt_setup(BrtSmem& S, const unsigned char* tcB, 
         S.twF[k] = tcTw[k];
         S.twI[k] = tcTw[1024 + k];
     }
-    if (tid < 32) tc_alloc<512>(&S.tmem);
+    if (tid >> 5 == kTcCompWarps) tc_alloc<512>(&S.tmem);
     if (tid == 0) {
-        mbar_init(&S.mbar, 1);
+        for (int s = 0; s < kTcSlots; s++) {
+            mbar_init(&S.full[s], 1);
+            mbar_init(&S.empty[s], 4);
+        }
+        for (int t = 0; t < kTcTiles; t++) mbar_init(&S.a2[t], 4);
+        mbar_init(&S.gate, kTcCompWarps);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     tc_fence_before();
@@ -309,7 +339,7 @@ __device__ __forceinline__ void brt_setup(BrtSmem& S, const unsigned char* tcB, 
 __device__ __forceinline__ void brt_teardown(BrtSmem& S) {
     tc_fence_before();
     __syncthreads();
-    if (threadIdx.x < 32) tc_dealloc<512>(S.tmem);
+    if (threadIdx.x >> 5 == kTcCompWarps) tc_dealloc<512>(S.tmem);
 }
 
 // ---- the blind-rotation kernel: a1 linear combination, a2 mod switch, a3 ACC init, a4 630 CMux, a5 extract ---
@@ -321,9 +351,9 @@ __global__ void __launch_bounds__(kTcThreads, 1) brt_kernel(BrArgs A, const uint
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int lane0 = blockIdx.x * kTcG;
     brt_setup(S, tcB, tcTw);
-    // a1 + a2: 6 warps per lane
-    {
-        const int g = warp / 6, w6 = warp % 6;
+    // a1 + a2: 3 compute warps per lane
+    if (warp < kTcCompWarps) {
+        const int g = warp / 3, w3 = warp % 3;
         const int gl = lane0 + g;
         LaneDesc d = {0, -1, 0, 0, 0u, 0u, 0u, 0u};
         if (gl < A.nlanes) d = A.lanes[gl];
@@ -332,7 +362,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) brt_kernel(BrArgs A, const uint
         const uint32_t* s1 = sb == 0 ? A.src0 : (sb == 1 ? A.src1 : A.src2);
         const uint32_t* pa = s0 + (int64_t)d.ia * A.src_stride;
         const uint32_t* pb = d.ib >= 0 ? s1 + (int64_t)d.ib * A.src_stride : nullptr;
-        for (int w = w6 * 32 + lane; w <= kn; w += 192) {
+        for (int w = w3 * 32 + lane; w <= kn; w += 96) {
             uint32_t v = (gl < A.nlanes) ? (uint32_t)d.wa * __ldg(pa + w) : 0u;
             if (pb) v += (uint32_t)d.wb * __ldg(pb + w);
             if (w == kn) v += d.cst;
@@ -348,14 +378,23 @@ __global__ void __launch_bounds__(kTcThreads, 1) brt_kernel(BrArgs A, const uint
         S.acc[gg][1][c] = ((c + bbar) & (kTwoN - 1)) < (uint32_t)kN ? kMu : (uint32_t)(0u - kMu);
     }
     __syncthreads();
-    uint32_t phase = 0;
-    for (int i = 0; i < kn; i++) {
-        brt_digits(S, i);
-        brt_cmux_tail(S, bk4 + (size_t)i * kN * kBk4Rec, phase);
+    uint32_t k = 0;
+    if (warp == kTcCompWarps) {
+        if (lane == 0) {
+            uint32_t gph = 0, aph = 0;
+            for (int i = 0; i < kn; i++) brt_mma_step(S, k, gph, aph);
+        }
+        __syncwarp();
+    } else {
+        for (int i = 0; i < kn; i++) {
+            brt_digits(S, i);
+            brt_comp_step(S, bk4 + (size_t)i * kN * kBk4Rec, k);
+        }
     }
+    __syncthreads();
     // a5: sample extraction, index 0 (C8)
-    for (int k = tid; k < kTcG * (kN + 1); k += kTcThreads) {
-        const int g = k / (kN + 1), j = k % (kN + 1);
+    for (int e = tid; e < kTcG * (kN + 1); e += kTcThreads) {
+        const int g = e / (kN + 1), j = e % (kN + 1);
         const int gl = lane0 + g;
         if (gl >= A.nlanes) continue;
         uint32_t v;
@@ -367,7 +406,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) brt_kernel(BrArgs A, const uint
     brt_teardown(S);
 }
 
-// ---- diagnostic: res[g][q] = sum_r d[g][r] (x) polys[r][q] mod 2^32 through one CMux tail (acc starts at 0) --
+// ---- diagnostic: res[g][q] = sum_r d[g][r] (x) polys[r][q] mod 2^32 through one CMux step (acc starts at 0) --
 __global__ void __launch_bounds__(kTcThreads, 1) brt_muladd_kernel(const int32_t* __restrict__ digits,
                                                                     const uint32_t* __restrict__ bk4,
                                                                     const unsigned char* __restrict__ tcB,
@@ -375,17 +414,28 @@ __global__ void __launch_bounds__(kTcThreads, 1) brt_muladd_kernel(const int32_t
                                                                     uint32_t* __restrict__ res) {
     extern __shared__ __align__(1024) unsigned char brt_smem[];
     BrtSmem& S = *reinterpret_cast<BrtSmem*>(brt_smem);
-    const int tid = threadIdx.x;
+    const int tid = threadIdx.x, warp = tid >> 5;
     brt_setup(S, tcB, tcTw);
-    for (int k = tid; k < kTcG * 2 * kN; k += kTcThreads) (&S.acc[0][0][0])[k] = 0u;
-    // digits [g][r][1024] -> A1 row (g*6 + r)*32 + k2, K byte k1
+    for (int e = tid; e < kTcG * 2 * kN; e += kTcThreads) (&S.acc[0][0][0])[e] = 0u;
+    // digits [g][r][1024] -> tile P / 4, row (P % 4)*32 + k2, K byte k1
     for (int e = tid; e < kTcPolys * kN; e += kTcThreads) {
         const int P = e / kN, c = e % kN, k1 = c >> 5, k2 = c & 31;
-        S.A1[tc_off(P * 32 + k2, k1, kA1Lbo, kA1Sbo)] = (unsigned char)(digits[e] & 0xFF);
+        S.op[(P >> 2) * kOpTile + tc_off((P & 3) * 32 + k2, k1, kA1Lbo, kA1Sbo)] = (unsigned char)(digits[e] & 0xFF);
     }
-    uint32_t phase = 0;
-    brt_cmux_tail(S, bk4, phase);
-    for (int k = tid; k < kTcG * 2 * kN; k += kTcThreads) res[k] = (&S.acc[0][0][0])[k];
+    fence_async_smem();
+    __syncthreads();
+    uint32_t k = 0;
+    if (warp == kTcCompWarps) {
+        if ((tid & 31) == 0) {
+            uint32_t gph = 0, aph = 0;
+            brt_mma_step(S, k, gph, aph);
+        }
+        __syncwarp();
+    } else {
+        brt_comp_step(S, bk4, k);
+    }
+    __syncthreads();
+    for (int e = tid; e < kTcG * 2 * kN; e += kTcThreads) res[e] = (&S.acc[0][0][0])[e];
     brt_teardown(S);
 }
 

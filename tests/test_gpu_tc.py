@@ -48,16 +48,16 @@ def test_tc_muladd_equals_schoolbook(ctx):
     import oracle as O
     rng = np.random.default_rng(5)
     M32 = 1 << 32
-    cases = [(rng.integers(-64, 64, (2, 6, 1024)), rng.integers(0, M32, (6, 2, 1024), dtype=np.uint64)),
-             (np.full((2, 6, 1024), -64), np.full((6, 2, 1024), M32 - 1, np.uint64)),
-             (np.stack([np.full((6, 1024), 63), np.full((6, 1024), -64)]), np.full((6, 2, 1024), 1 << 31, np.uint64)),
-             (np.zeros((2, 6, 1024), int), rng.integers(0, M32, (6, 2, 1024), dtype=np.uint64))]
+    cases = [(rng.integers(-64, 64, (4, 6, 1024)), rng.integers(0, M32, (6, 2, 1024), dtype=np.uint64)),
+             (np.full((4, 6, 1024), -64), np.full((6, 2, 1024), M32 - 1, np.uint64)),
+             (np.stack([np.full((6, 1024), 63), np.full((6, 1024), -64)] * 2), np.full((6, 2, 1024), 1 << 31, np.uint64)),
+             (np.zeros((4, 6, 1024), int), rng.integers(0, M32, (6, 2, 1024), dtype=np.uint64))]
     for d, b in cases:
         d32 = d.astype(np.int32)
         b32 = b.astype(np.uint32)
         got = ctx.tc_muladd(torch.from_numpy(d32).cuda(), torch.from_numpy(b32.view(np.int32)).cuda())
         got = got.cpu().numpy().view(np.uint32)
-        for g in range(2):
+        for g in range(4):
             for q in range(2):
                 want = np.zeros(1024, np.uint32)
                 for r in range(6):
