@@ -20,15 +20,16 @@
 // u8 x u8 (digits: s8 x u8) with K = 32 (digits) or 128 and N = 128 (4 limbs x 32), and the CUDA cores only
 // recombine the 4 limbs (one Shoup product by 2^16) and apply the twiddles.
 //
-// Structure (one CTA per SM, G = 4 lanes = bootstraps, accumulators resident in shared memory for all n = 630
-// CMux steps).  A CMux step is 4 GEMM stages x 6 tile jobs (a tile = 4 polynomials = 128 rows):
-//   digits (all compute warps) -> GEMM1 -> ep1 (limbs, twiddle) -> GEMM2 -> ep2 (limbs) -> MAC (all compute
-//   warps; each NTT-domain BK word read once for the 4 lanes) -> GEMM3 -> ep3 (limbs, twiddle) -> GEMM4 -> ep4
-//   (limbs, lift, ACC +=).
-// Warp 12 issues the MMAs (one thread) into a ring of 4 TMEM slots (128 columns each) and runs ahead of the 12
-// compute warps (3 quads of 4 warps, one warp per TMEM lane quadrant); a quad takes every third tile job of a
-// stage.  mbarriers: full[slot] (MMA commit -> epilogue), empty[slot] (4 epilogue warps -> MMA), a2[tile] (ep1
-// wrote GEMM2's operand tile), gate (all 12 compute warps done with digits / MAC / ep3).
+// Structure: one CTA per SM holds two independent groups of G = 2 lanes (bootstraps); each group's accumulators
+// stay in shared memory for all n = 630 CMux steps.  A group's CMux step is 4 GEMM stages x 3 tile jobs (a tile
+// = 4 polynomials = 128 rows of the M = 128 MMA):
+//   digits -> GEMM1 -> ep1 (limbs, twiddle) -> GEMM2 -> ep2 (limbs) -> MAC (each NTT-domain BK word read once
+//   for the group's 2 lanes) -> GEMM3 -> ep3 (limbs, twiddle) -> GEMM4 -> ep4 (limbs, lift, ACC +=).
+// Per group: one MMA warp (one thread issues) fills a ring of 2 TMEM slots (128 columns each) and runs ahead of
+// 8 compute warps (2 quads; a warp reads its TMEM lane quadrant, the two quads split a slot's columns).  The two
+// groups drift apart, so one group's MAC and digit phases (CUDA cores and L2 only) overlap the other group's
+// GEMMs and epilogues.  mbarriers per group: full[slot] (MMA commit -> epilogue), empty[slot] (8 epilogue warps
+// -> MMA), a2[tile] (ep1 wrote GEMM2's operand tile), gate (all 8 compute warps done with digits / MAC / ep3).
 #include <cstring>
 
 #include "tb_kernels.cuh"
@@ -37,13 +38,16 @@
 
 namespace tb {
 
-constexpr int kTcG = 4;                       // lanes per CTA
-constexpr int kTcPolys = 6 * kTcG;            // polynomials per transform stage (24 = 6 tiles of 4)
+constexpr int kTcG = 2;                       // lanes per group
+constexpr int kTcGroups = 2;                  // groups per CTA
+constexpr int kTcLanes = kTcG * kTcGroups;    // lanes per CTA
+constexpr int kTcPolys = 6 * kTcG;            // polynomials per transform stage of a group (12 = 3 tiles of 4)
 constexpr int kTcTiles = kTcPolys / 4;
-constexpr int kTcCompWarps = 12;
-constexpr int kTcCompThreads = 32 * kTcCompWarps;
-constexpr int kTcThreads = kTcCompThreads + 32;         // + the MMA warp
-constexpr int kTcSlots = 4;                              // TMEM ring: 4 x 128 columns
+constexpr int kTcGWarps = 8;                  // compute warps per group
+constexpr int kTcGThreads = 32 * kTcGWarps;
+constexpr int kTcCompWarps = kTcGWarps * kTcGroups;
+constexpr int kTcThreads = 32 * (kTcCompWarps + kTcGroups);   // + one MMA warp per group
+constexpr int kTcSlots = 2;                              // TMEM ring per group: 2 x 128 columns
 // shared-memory operand layouts (K-major core matrices, tb_tc.cuh)
 constexpr uint32_t kA1Lbo = 128, kA1Sbo = 256;          // digits: 128 rows x 32 B per tile (at the tile's start)
 constexpr uint32_t kOpLbo = 144, kOpSbo = 8 * 144;      // 30-bit operands: 128 rows x 128 B per tile (padded)
@@ -52,14 +56,17 @@ constexpr uint32_t kB1Bytes = 128 * 32, kBBytes = 128 * 128;
 constexpr uint32_t kTcBTotal = kB1Bytes + 3 * kBBytes;  // B1 (W1 bytes), B2 (W2'), B3 (V2'), B4 (V1')
 constexpr int kBk4Rec = 36;                              // NTT-domain BK record per coefficient: [r][o]
 
-struct BrtSmem {
-    unsigned char B[kTcBTotal];                  // constant B operands (dense: LBO 128)
+struct BrtGroup {
     unsigned char op[kTcTiles * kOpTile];        // per tile: A1 | A2 | MAC in / out = A3 | A4 (stage-aliased)
-    uint2 twF[32 * 32];                          // [j1][k2] (psi^((2 j1 + 1) k2), Shoup)
-    uint2 twI[32 * 32];                          // [k2][j1] (psi^(-(2 j1 + 1) k2), Shoup)
     uint32_t acc[kTcG][2][kN];
     uint16_t bar[kTcG][kn + 2];
     uint64_t full[kTcSlots], empty[kTcSlots], a2[kTcTiles], gate;
+};
+struct BrtSmem {
+    unsigned char B[kTcBTotal];                  // constant B operands (dense: LBO 128)
+    uint2 twF[32 * 32];                          // [j1][k2] (psi^((2 j1 + 1) k2), Shoup)
+    uint2 twI[32 * 32];                          // [k2][j1] (psi^(-(2 j1 + 1) k2), Shoup)
+    BrtGroup grp[kTcGroups];
     uint32_t tmem;
 };
 
@@ -81,26 +88,30 @@ __device__ __forceinline__ uint32_t limbs_s(uint32_t y0, uint32_t y1, uint32_t y
 __device__ __forceinline__ void mbar_arrive(uint64_t* b) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
 }
-__device__ __forceinline__ void comp_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kTcCompThreads) : "memory"); }
+// named barrier of a group's compute warps (ids 1, 2)
+__device__ __forceinline__ void grp_sync(int grp) {
+    asm volatile("bar.sync %0, %1;" ::"r"(1 + grp), "n"(kTcGThreads) : "memory");
+}
 
 // byte offset of (row, 32-bit word) of an operand tile
 __host__ __device__ constexpr uint32_t opw(uint32_t row, uint32_t word) { return tc_off(row, 4 * word, kOpLbo, kOpSbo); }
 
-// ---- MMA warp: the static job sequence of one CMux step (stage s, tile t), job counter k across steps -------
-__device__ __forceinline__ void brt_mma_step(BrtSmem& S, uint32_t& k, uint32_t& gate_ph, uint32_t& a2_ph) {
-    const uint32_t sB = smem_u32(S.B), sOp = smem_u32(S.op);
+// ---- MMA warp of a group: the static job sequence of one CMux step (stage s, tile t); k counts jobs ---------
+__device__ __forceinline__ void brt_mma_step(BrtSmem& S, BrtGroup& G, uint32_t tmem, uint32_t& k, uint32_t& gate_ph,
+                                             uint32_t& a2_ph) {
+    const uint32_t sB = smem_u32(S.B), sOp = smem_u32(G.op);
     constexpr uint32_t id_s = tc_idesc_i8(128, 128, true, false), id_u = tc_idesc_i8(128, 128, false, false);
     for (int s = 0; s < 4; s++) {
         if (s != 1) {                                   // digits / MAC / ep3 of every compute warp done
-            mbar_wait(&S.gate, gate_ph);
+            mbar_wait(&G.gate, gate_ph);
             gate_ph ^= 1;
         }
         for (int t = 0; t < kTcTiles; t++, k++) {
             const uint32_t slot = k % kTcSlots;
-            if (s == 1) mbar_wait(&S.a2[t], a2_ph);     // ep1 wrote this tile's GEMM2 operand
-            if (k >= kTcSlots) mbar_wait(&S.empty[slot], ((k / kTcSlots) - 1) & 1);
+            if (s == 1) mbar_wait(&G.a2[t], a2_ph);     // ep1 wrote this tile's GEMM2 operand
+            if (k >= kTcSlots) mbar_wait(&G.empty[slot], ((k / kTcSlots) - 1) & 1);
             tc_fence_after();
-            const uint32_t d = S.tmem + 128 * slot;
+            const uint32_t d = tmem + 128 * slot;
             const uint32_t a = sOp + t * kOpTile;
             if (s == 0) {
                 tc_mma_i8(d, tc_sdesc(a, kA1Lbo, kA1Sbo), tc_sdesc(sB, 128, 256), id_s, 0);
@@ -111,97 +122,92 @@ __device__ __forceinline__ void brt_mma_step(BrtSmem& S, uint32_t& k, uint32_t& 
                     tc_mma_i8(d, tc_sdesc(a + 2 * q * kOpLbo, kOpLbo, kOpSbo), tc_sdesc(bb + 2 * q * 128, 128, 1024),
                               id_u, q > 0);
             }
-            tc_commit(smem_u32(&S.full[slot]));
+            tc_commit(smem_u32(&G.full[slot]));
         }
         if (s == 1) a2_ph ^= 1;
     }
 }
 
-// ---- compute warps ---------------------------------------------------------------------------------------
-// digits of (X^abar - 1) ACC for the 4 lanes -> A1 (a4.1).  Task (g, bloc, k2, h): coefficients
+// ---- compute warps of a group ----------------------------------------------------------------------------
+// digits of (X^abar - 1) ACC for the group's 2 lanes -> A1 (a4.1).  Thread (g, bloc, h, k2): coefficients
 // c = 32 (16 h + u) + k2, u < 16; digit jd of polynomial P = g*6 + bloc*3 + jd goes to tile P / 4, row
 // (P % 4)*32 + k2, K bytes 16 h .. 16 h + 15 (one 16-byte store)
-__device__ __forceinline__ void brt_digits(BrtSmem& S, int i) {
-    for (int task = threadIdx.x; task < kTcG * 2 * 32 * 2; task += kTcCompThreads) {
-        const int k2 = task & 31, h = (task >> 5) & 1, bloc = (task >> 6) & 1, g = task >> 7;
-        const uint32_t ab = S.bar[g][i];
-        const uint32_t* acc = S.acc[g][bloc];
-        uint32_t d[3][4] = {};
+__device__ __forceinline__ void brt_digits(BrtGroup& G, int i, int gt) {
+    const int k2 = gt & 31, h = (gt >> 5) & 1, bloc = (gt >> 6) & 1, g = gt >> 7;
+    const uint32_t ab = G.bar[g][i];
+    const uint32_t* acc = G.acc[g][bloc];
+    uint32_t d[3][4] = {};
 #pragma unroll
-        for (int u = 0; u < 16; u++) {
-            const uint32_t c = 32u * (16 * h + u) + k2;
-            const uint32_t mm = (c - ab) & (kTwoN - 1);
-            const uint32_t src = acc[mm & (kN - 1)];
-            const uint32_t rot = mm < (uint32_t)kN ? src : 0u - src;
-            const uint32_t x = rot - acc[c] + c_misc[3];             // (X^abar - 1) ACC + decomposition offset
-#pragma unroll
-            for (int jd = 0; jd < 3; jd++) {
-                const uint32_t dig = ((x >> (32 - kBgbit * (jd + 1))) & 127u) - 64u;   // digit in [-64, 63]
-                d[jd][u >> 2] |= (dig & 0xFFu) << (8 * (u & 3));
-            }
-        }
+    for (int u = 0; u < 16; u++) {
+        const uint32_t c = 32u * (16 * h + u) + k2;
+        const uint32_t mm = (c - ab) & (kTwoN - 1);
+        const uint32_t src = acc[mm & (kN - 1)];
+        const uint32_t rot = mm < (uint32_t)kN ? src : 0u - src;
+        const uint32_t x = rot - acc[c] + c_misc[3];             // (X^abar - 1) ACC + decomposition offset
 #pragma unroll
         for (int jd = 0; jd < 3; jd++) {
-            const int P = g * 6 + bloc * 3 + jd;
-            *reinterpret_cast<uint4*>(S.op + (P >> 2) * kOpTile + tc_off((P & 3) * 32 + k2, 16 * h, kA1Lbo, kA1Sbo)) =
-                make_uint4(d[jd][0], d[jd][1], d[jd][2], d[jd][3]);
+            const uint32_t dig = ((x >> (32 - kBgbit * (jd + 1))) & 127u) - 64u;   // digit in [-64, 63]
+            d[jd][u >> 2] |= (dig & 0xFFu) << (8 * (u & 3));
         }
+    }
+#pragma unroll
+    for (int jd = 0; jd < 3; jd++) {
+        const int P = g * 6 + bloc * 3 + jd;
+        *reinterpret_cast<uint4*>(G.op + (P >> 2) * kOpTile + tc_off((P & 3) * 32 + k2, 16 * h, kA1Lbo, kA1Sbo)) =
+            make_uint4(d[jd][0], d[jd][1], d[jd][2], d[jd][3]);
     }
 }
 
-// Where the MAC writes output o of lane g (and so where GEMM3 / ep3 / GEMM4 / ep4 find it): tile
-// (m = o % 3) * 2 + g / 2, quadrant (g % 2) * 2 + q (q = o / 3).  Then GEMM3's tile (m, h) holds exactly the
-// polynomials whose ep3 output fills A4 tile (m, h): ep3 rewrites only the tile it has just consumed.
-__device__ __forceinline__ int mac_out_tile(int g, int o) { return (o % 3) * 2 + (g >> 1); }
-__device__ __forceinline__ int mac_out_quad(int g, int o) { return (g & 1) * 2 + o / 3; }
+// Where the MAC writes output o of lane g (and so where GEMM3 / ep3 / GEMM4 / ep4 find it): tile m = o % 3,
+// quadrant g * 2 + q (q = o / 3).  GEMM3's tile m then holds exactly the polynomials whose ep3 output fills A4
+// tile m (rows (g, q, k2)): ep3 rewrites only the tile it has just consumed, and ep4 of tile m adds part m.
 
-// The compute warps' part of one CMux step; k = job counter (same sequence as the MMA warp)
-__device__ __forceinline__ void brt_comp_step(BrtSmem& S, const uint32_t* __restrict__ bk4, uint32_t& k,
-                                              uint32_t* __restrict__ res_debug = nullptr) {
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int quad = warp >> 2, qd = warp & 3;
-    const uint32_t tq = S.tmem + ((uint32_t)(32 * qd) << 16);     // this warp's TMEM lane quadrant
-    // digits were written by the caller; publish them to the MMA warp
-    fence_async_smem();
+// One CMux step of a group's compute warps (the digits are in A1); k = job counter (same as the MMA warp's)
+__device__ __forceinline__ void brt_comp_step(BrtSmem& S, BrtGroup& G, uint32_t tmem, int grp, int gw,
+                                              const uint32_t* __restrict__ bk4, uint32_t& k) {
+    const int lane = threadIdx.x & 31;
+    const int hq = gw >> 2, qd = gw & 3;                 // column half (quad) and TMEM lane quadrant
+    const uint32_t tq = tmem + ((uint32_t)(32 * qd) << 16) + 64 * hq;
+    fence_async_smem();                                  // publish the digits to the MMA warp
     __syncwarp();
-    if (lane == 0) mbar_arrive(&S.gate);
-    // ---- ep1: job (0, t), t % 3 == quad: thread (P = 4t + qd, k2 = lane): C[j1][k2] -> A2 row (qd, j1) word k2
-    for (int t = quad; t < kTcTiles; t += 3) {
+    if (lane == 0) mbar_arrive(&G.gate);
+    // ---- ep1: tile t, thread (P = 4t + qd, k2 = lane), j1 in this quad's half: C[j1][k2] -> A2 row (qd, j1)
+    for (int t = 0; t < kTcTiles; t++) {
         const uint32_t kk = k + t, slot = kk % kTcSlots;
-        mbar_wait(&S.full[slot], (kk / kTcSlots) & 1);
+        mbar_wait(&G.full[slot], (kk / kTcSlots) & 1);
         tc_fence_after();
-        unsigned char* base = S.op + t * kOpTile + opw(qd * 32, lane);
-        const uint2* tw = S.twF + lane;
+        unsigned char* base = G.op + t * kOpTile + opw(qd * 32 + 16 * hq, lane);
+        const uint2* tw = S.twF + 32 * 16 * hq + lane;
 #pragma unroll
-        for (int jc = 0; jc < 8; jc++) {
+        for (int jc = 0; jc < 4; jc++) {
             uint32_t v[16];
             tc_ld16(tq + 128 * slot + 16 * jc, v);
             tc_wait_ld();
 #pragma unroll
             for (int u = 0; u < 4; u++) {
-                const int j1 = 4 * jc + u;
+                const int j = 4 * jc + u;                  // j1 = 16 hq + j
                 const uint32_t x = limbs_s(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3]);
-                const uint2 w = tw[32 * j1];
-                *reinterpret_cast<uint32_t*>(base + (j1 >> 3) * kOpSbo + (j1 & 7) * 16) = shoup_mul(x, w.x, w.y);
+                const uint2 w = tw[32 * j];
+                *reinterpret_cast<uint32_t*>(base + (j >> 3) * kOpSbo + (j & 7) * 16) = shoup_mul(x, w.x, w.y);
             }
         }
         fence_async_smem();
         tc_fence_before();
         __syncwarp();
         if (lane == 0) {
-            mbar_arrive(&S.empty[slot]);
-            mbar_arrive(&S.a2[t]);
+            mbar_arrive(&G.empty[slot]);
+            mbar_arrive(&G.a2[t]);
         }
     }
     k += kTcTiles;
-    // ---- ep2: job (1, t): thread (P = 4t + qd, j1 = lane): A[j1 + 32 j2] in [0, 2p) -> row (qd, j1) words j2
-    for (int t = quad; t < kTcTiles; t += 3) {
+    // ---- ep2: tile t, thread (P = 4t + qd, j1 = lane), j2 in this quad's half: A[j1 + 32 j2] in [0, 2p)
+    for (int t = 0; t < kTcTiles; t++) {
         const uint32_t kk = k + t, slot = kk % kTcSlots;
-        mbar_wait(&S.full[slot], (kk / kTcSlots) & 1);
+        mbar_wait(&G.full[slot], (kk / kTcSlots) & 1);
         tc_fence_after();
-        unsigned char* base = S.op + t * kOpTile + opw(qd * 32 + lane, 0);
+        unsigned char* base = G.op + t * kOpTile + opw(qd * 32 + lane, 16 * hq);
 #pragma unroll
-        for (int c = 0; c < 8; c++) {
+        for (int c = 0; c < 4; c++) {
             uint32_t v[16];
             tc_ld16(tq + 128 * slot + 16 * c, v);
             tc_wait_ld();
@@ -214,17 +220,16 @@ __device__ __forceinline__ void brt_comp_step(BrtSmem& S, const uint32_t* __rest
         }
         tc_fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(&S.empty[slot]);
+        if (lane == 0) mbar_arrive(&G.empty[slot]);
     }
     k += kTcTiles;
-    comp_sync();                                    // every ep2 tile written
-    // ---- MAC: coefficient (j1, j2) of the 4 lanes, M_o = sum_r A_r BK4[r][o] (a4.3); each BK word read once
+    grp_sync(grp);                                       // every ep2 tile of the group written
+    // ---- MAC: coefficient (j1, j2 = lane) of the 2 lanes, M_o = sum_r A_r BK4[r][o] (a4.3), in place per thread
     {
         const uint32_t R = c_misc[0], Rp = c_misc[1];
-        const uint32_t lanew = (lane >> 2) * kOpLbo + (lane & 3) * 4;     // word j2 = lane within a row
-        for (int j1 = warp; j1 < 32; j1 += kTcCompWarps) {
-            const int pos = j1 * 32 + lane;
-            const uint4* rec = reinterpret_cast<const uint4*>(bk4 + (size_t)pos * kBk4Rec);
+        const uint32_t lanew = (lane >> 2) * kOpLbo + (lane & 3) * 4;
+        for (int j1 = gw; j1 < 32; j1 += kTcGWarps) {
+            const uint4* rec = reinterpret_cast<const uint4*>(bk4 + (size_t)(j1 * 32 + lane) * kBk4Rec);
             uint32_t B[kBk4Rec];
 #pragma unroll
             for (int q = 0; q < kBk4Rec / 4; q++) {
@@ -238,7 +243,7 @@ __device__ __forceinline__ void brt_comp_step(BrtSmem& S, const uint32_t* __rest
 #pragma unroll
                 for (int r = 0; r < 6; r++) {
                     const int P = g * 6 + r;
-                    D[g][r] = *reinterpret_cast<const uint32_t*>(S.op + (P >> 2) * kOpTile + (P & 3) * 4 * kOpSbo + rowoff);
+                    D[g][r] = *reinterpret_cast<const uint32_t*>(G.op + (P >> 2) * kOpTile + (P & 3) * 4 * kOpSbo + rowoff);
                 }
 #pragma unroll
             for (int g = 0; g < kTcG; g++)
@@ -248,88 +253,90 @@ __device__ __forceinline__ void brt_comp_step(BrtSmem& S, const uint32_t* __rest
 #pragma unroll
                     for (int r = 0; r < 6; r++) s += (uint64_t)D[g][r] * B[r * 6 + o];
                     const uint32_t hi = (uint32_t)(s >> 32), lo = (uint32_t)s;
-                    *reinterpret_cast<uint32_t*>(S.op + mac_out_tile(g, o) * kOpTile + mac_out_quad(g, o) * 4 * kOpSbo +
-                                                 rowoff) = red_2p(shoup_mul(hi, R, Rp) + (lo - (lo >> 30) * kP));
+                    *reinterpret_cast<uint32_t*>(G.op + (o % 3) * kOpTile + (g * 2 + o / 3) * 4 * kOpSbo + rowoff) =
+                        red_2p(shoup_mul(hi, R, Rp) + (lo - (lo >> 30) * kP));
                 }
         }
     }
-    fence_async_smem();                             // (the MAC is in place per thread: one thread owns (j1, j2))
+    fence_async_smem();
     __syncwarp();
-    if (lane == 0) mbar_arrive(&S.gate);
-    // ---- ep3: job (2, t = m*2 + h): thread (quadrant qd = (g%2)*2 + q, j1 = lane): D[j1][k2] -> E -> A4 tile t
-    // row (qd, k2) word j1 (the tile GEMM3 just consumed)
-    for (int t = quad; t < kTcTiles; t += 3) {
+    if (lane == 0) mbar_arrive(&G.gate);
+    // ---- ep3: tile m, thread (quadrant qd = g*2 + q, j1 = lane), k2 in this quad's half: D[j1][k2] -> E -> A4
+    // tile m row (qd, k2) word j1 (the tile GEMM3 just consumed)
+    for (int t = 0; t < kTcTiles; t++) {
         const uint32_t kk = k + t, slot = kk % kTcSlots;
-        mbar_wait(&S.full[slot], (kk / kTcSlots) & 1);
+        mbar_wait(&G.full[slot], (kk / kTcSlots) & 1);
         tc_fence_after();
-        unsigned char* base = S.op + t * kOpTile + opw(qd * 32, lane);
-        const uint2* tw = S.twI + lane;
+        unsigned char* base = G.op + t * kOpTile + opw(qd * 32 + 16 * hq, lane);
+        const uint2* tw = S.twI + 32 * 16 * hq + lane;
 #pragma unroll
-        for (int c = 0; c < 8; c++) {
+        for (int c = 0; c < 4; c++) {
             uint32_t v[16];
             tc_ld16(tq + 128 * slot + 16 * c, v);
             tc_wait_ld();
 #pragma unroll
             for (int u = 0; u < 4; u++) {
-                const int k2 = 4 * c + u;
+                const int j = 4 * c + u;                  // k2 = 16 hq + j
                 const uint32_t x = limbs_u(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3]);
-                const uint2 w = tw[32 * k2];
-                *reinterpret_cast<uint32_t*>(base + (k2 >> 3) * kOpSbo + (k2 & 7) * 16) = shoup_mul(x, w.x, w.y);
+                const uint2 w = tw[32 * j];
+                *reinterpret_cast<uint32_t*>(base + (j >> 3) * kOpSbo + (j & 7) * 16) = shoup_mul(x, w.x, w.y);
             }
         }
         fence_async_smem();
         tc_fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(&S.empty[slot]);
+        if (lane == 0) mbar_arrive(&G.empty[slot]);
     }
     k += kTcTiles;
-    // GEMM4 needs every A4 tile: ep3 of every quad done
     __syncwarp();
-    if (lane == 0) mbar_arrive(&S.gate);
-    // ---- ep4: job (3, t = m*2 + h): thread (g = 2h + qd/2, q = qd%2, k2 = lane): part m of N a[32 k1 + k2] ->
-    // centred lift, << 11 m, added into ACC[g][q] (a4.4; the three part jobs of (g, q) add atomically)
-    for (int t = quad; t < kTcTiles; t += 3) {
+    if (lane == 0) mbar_arrive(&G.gate);                 // GEMM4 needs every A4 tile
+    // ---- ep4: tile m, thread (g = qd / 2, q = qd % 2, k2 = lane), k1 in this quad's half: part m of
+    // N a[32 k1 + k2] -> centred lift, << 11 m, added into ACC[g][q] (a4.4; the parts are added one tile after
+    // the other, the quads own disjoint k1)
+    for (int t = 0; t < kTcTiles; t++) {
         const uint32_t kk = k + t, slot = kk % kTcSlots;
-        mbar_wait(&S.full[slot], (kk / kTcSlots) & 1);
+        mbar_wait(&G.full[slot], (kk / kTcSlots) & 1);
         tc_fence_after();
-        const int m = t >> 1, g = 2 * (t & 1) + (qd >> 1), q = qd & 1;
-        uint32_t* acc = &S.acc[g][q][lane];
+        uint32_t* acc = &G.acc[qd >> 1][qd & 1][32 * 16 * hq + lane];
 #pragma unroll
-        for (int c = 0; c < 8; c++) {
+        for (int c = 0; c < 4; c++) {
             uint32_t v[16];
             tc_ld16(tq + 128 * slot + 16 * c, v);
             tc_wait_ld();
 #pragma unroll
             for (int u = 0; u < 4; u++) {
-                const int k1 = 4 * c + u;
+                const int j = 4 * c + u;                  // k1 = 16 hq + j
                 const uint32_t a = lift_centred(red_2p(limbs_u(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3])));
-                atomicAdd(acc + 32 * k1, a << (11 * m));
+                acc[32 * j] += a << (11 * t);
             }
         }
         tc_fence_before();
         __syncwarp();
-        if (lane == 0) mbar_arrive(&S.empty[slot]);
+        if (lane == 0) mbar_arrive(&G.empty[slot]);
     }
     k += kTcTiles;
-    comp_sync();                                    // ACC complete before the next step's digits
+    grp_sync(grp);                                       // ACC complete before the next step's digits
 }
 
 __device__ __forceinline__ void brt_setup(BrtSmem& S, const unsigned char* tcB, const uint2* tcTw) {
     const int tid = threadIdx.x;
-    for (int k = tid; k < (int)(kTcBTotal / 16); k += kTcThreads)
-        reinterpret_cast<uint4*>(S.B)[k] = __ldg(reinterpret_cast<const uint4*>(tcB) + k);
-    for (int k = tid; k < 32 * 32; k += kTcThreads) {
-        S.twF[k] = tcTw[k];
-        S.twI[k] = tcTw[1024 + k];
+    for (int e = tid; e < (int)(kTcBTotal / 16); e += kTcThreads)
+        reinterpret_cast<uint4*>(S.B)[e] = __ldg(reinterpret_cast<const uint4*>(tcB) + e);
+    for (int e = tid; e < 32 * 32; e += kTcThreads) {
+        S.twF[e] = tcTw[e];
+        S.twI[e] = tcTw[1024 + e];
     }
     if (tid >> 5 == kTcCompWarps) tc_alloc<512>(&S.tmem);
     if (tid == 0) {
-        for (int s = 0; s < kTcSlots; s++) {
-            mbar_init(&S.full[s], 1);
-            mbar_init(&S.empty[s], 4);
+        for (int gi = 0; gi < kTcGroups; gi++) {
+            BrtGroup& G = S.grp[gi];
+            for (int s = 0; s < kTcSlots; s++) {
+                mbar_init(&G.full[s], 1);
+                mbar_init(&G.empty[s], kTcGWarps);
+            }
+            for (int t = 0; t < kTcTiles; t++) mbar_init(&G.a2[t], kTcGWarps);
+            mbar_init(&G.gate, kTcGWarps);
         }
-        for (int t = 0; t < kTcTiles; t++) mbar_init(&S.a2[t], 4);
-        mbar_init(&S.gate, kTcCompWarps);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     tc_fence_before();
@@ -342,6 +349,28 @@ __device__ __forceinline__ void brt_teardown(BrtSmem& S) {
     if (threadIdx.x >> 5 == kTcCompWarps) tc_dealloc<512>(S.tmem);
 }
 
+// the 630 CMux steps of the CTA: warps [8 grp, 8 grp + 8) compute for group grp, warp 16 + grp issues its MMAs
+template <bool kDiag>
+__device__ __forceinline__ void brt_main(BrtSmem& S, const uint32_t* __restrict__ bk4, int nsteps) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    uint32_t k = 0;
+    if (warp >= kTcCompWarps) {
+        const int grp = warp - kTcCompWarps;
+        if (lane == 0) {
+            uint32_t gph = 0, aph = 0;
+            for (int i = 0; i < nsteps; i++) brt_mma_step(S, S.grp[grp], S.tmem + 256 * grp, k, gph, aph);
+        }
+        __syncwarp();
+    } else {
+        const int grp = warp / kTcGWarps, gw = warp % kTcGWarps;
+        BrtGroup& G = S.grp[grp];
+        for (int i = 0; i < nsteps; i++) {
+            if (!kDiag) brt_digits(G, i, threadIdx.x % kTcGThreads);
+            brt_comp_step(S, G, S.tmem + 256 * grp, grp, gw, bk4 + (size_t)i * kN * kBk4Rec, k);
+        }
+    }
+}
+
 // ---- the blind-rotation kernel: a1 linear combination, a2 mod switch, a3 ACC init, a4 630 CMux, a5 extract ---
 __global__ void __launch_bounds__(kTcThreads, 1) brt_kernel(BrArgs A, const uint32_t* __restrict__ bk4,
                                                              const unsigned char* __restrict__ tcB,
@@ -349,12 +378,12 @@ __global__ void __launch_bounds__(kTcThreads, 1) brt_kernel(BrArgs A, const uint
     extern __shared__ __align__(1024) unsigned char brt_smem[];
     BrtSmem& S = *reinterpret_cast<BrtSmem*>(brt_smem);
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int lane0 = blockIdx.x * kTcG;
+    const int lane0 = blockIdx.x * kTcLanes;
     brt_setup(S, tcB, tcTw);
-    // a1 + a2: 3 compute warps per lane
+    // a1 + a2: 4 compute warps per lane (lane L = grp * 2 + g)
     if (warp < kTcCompWarps) {
-        const int g = warp / 3, w3 = warp % 3;
-        const int gl = lane0 + g;
+        const int L = warp / 4, w4 = warp % 4;
+        const int gl = lane0 + L;
         LaneDesc d = {0, -1, 0, 0, 0u, 0u, 0u, 0u};
         if (gl < A.nlanes) d = A.lanes[gl];
         const uint32_t* s0 = (d.sel & 3u) == 0 ? A.src0 : ((d.sel & 3u) == 1 ? A.src1 : A.src2);
@@ -362,51 +391,42 @@ __global__ void __launch_bounds__(kTcThreads, 1) brt_kernel(BrArgs A, const uint
         const uint32_t* s1 = sb == 0 ? A.src0 : (sb == 1 ? A.src1 : A.src2);
         const uint32_t* pa = s0 + (int64_t)d.ia * A.src_stride;
         const uint32_t* pb = d.ib >= 0 ? s1 + (int64_t)d.ib * A.src_stride : nullptr;
-        for (int w = w3 * 32 + lane; w <= kn; w += 96) {
+        uint16_t* bar = S.grp[L / kTcG].bar[L % kTcG];
+        for (int w = w4 * 32 + lane; w <= kn; w += 128) {
             uint32_t v = (gl < A.nlanes) ? (uint32_t)d.wa * __ldg(pa + w) : 0u;
             if (pb) v += (uint32_t)d.wb * __ldg(pb + w);
             if (w == kn) v += d.cst;
-            S.bar[g][w] = (uint16_t)((v + (1u << 20)) >> 21);      // round(v 2N / 2^32) mod 2N (C5)
+            bar[w] = (uint16_t)((v + (1u << 20)) >> 21);      // round(v 2N / 2^32) mod 2N (C5)
         }
     }
     __syncthreads();
     // a3: ACC = (0, X^{-bbar} (mu, ..., mu))  (C6)
-    for (int k = tid; k < kTcG * kN; k += kTcThreads) {
-        const int gg = k / kN, c = k % kN;
-        const uint32_t bbar = S.bar[gg][kn];
-        S.acc[gg][0][c] = 0u;
-        S.acc[gg][1][c] = ((c + bbar) & (kTwoN - 1)) < (uint32_t)kN ? kMu : (uint32_t)(0u - kMu);
+    for (int e = tid; e < kTcLanes * kN; e += kTcThreads) {
+        const int L = e / kN, c = e % kN;
+        BrtGroup& G = S.grp[L / kTcG];
+        const uint32_t bbar = G.bar[L % kTcG][kn];
+        G.acc[L % kTcG][0][c] = 0u;
+        G.acc[L % kTcG][1][c] = ((c + bbar) & (kTwoN - 1)) < (uint32_t)kN ? kMu : (uint32_t)(0u - kMu);
     }
     __syncthreads();
-    uint32_t k = 0;
-    if (warp == kTcCompWarps) {
-        if (lane == 0) {
-            uint32_t gph = 0, aph = 0;
-            for (int i = 0; i < kn; i++) brt_mma_step(S, k, gph, aph);
-        }
-        __syncwarp();
-    } else {
-        for (int i = 0; i < kn; i++) {
-            brt_digits(S, i);
-            brt_comp_step(S, bk4 + (size_t)i * kN * kBk4Rec, k);
-        }
-    }
+    brt_main<false>(S, bk4, kn);
     __syncthreads();
     // a5: sample extraction, index 0 (C8)
-    for (int e = tid; e < kTcG * (kN + 1); e += kTcThreads) {
-        const int g = e / (kN + 1), j = e % (kN + 1);
-        const int gl = lane0 + g;
+    for (int e = tid; e < kTcLanes * (kN + 1); e += kTcThreads) {
+        const int L = e / (kN + 1), j = e % (kN + 1);
+        const int gl = lane0 + L;
         if (gl >= A.nlanes) continue;
+        const uint32_t(*acc)[kN] = S.grp[L / kTcG].acc[L % kTcG];
         uint32_t v;
-        if (j == 0) v = S.acc[g][0][0];
-        else if (j < kN) v = 0u - S.acc[g][0][kN - j];
-        else v = S.acc[g][1][0];
+        if (j == 0) v = acc[0][0];
+        else if (j < kN) v = 0u - acc[0][kN - j];
+        else v = acc[1][0];
         A.out[(int64_t)gl * A.out_stride + j] = v;
     }
     brt_teardown(S);
 }
 
-// ---- diagnostic: res[g][q] = sum_r d[g][r] (x) polys[r][q] mod 2^32 through one CMux step (acc starts at 0) --
+// ---- diagnostic: res[L][q] = sum_r d[L][r] (x) polys[r][q] mod 2^32 through one CMux step (acc starts at 0) --
 __global__ void __launch_bounds__(kTcThreads, 1) brt_muladd_kernel(const int32_t* __restrict__ digits,
                                                                     const uint32_t* __restrict__ bk4,
                                                                     const unsigned char* __restrict__ tcB,
@@ -414,28 +434,27 @@ __global__ void __launch_bounds__(kTcThreads, 1) brt_muladd_kernel(const int32_t
                                                                     uint32_t* __restrict__ res) {
     extern __shared__ __align__(1024) unsigned char brt_smem[];
     BrtSmem& S = *reinterpret_cast<BrtSmem*>(brt_smem);
-    const int tid = threadIdx.x, warp = tid >> 5;
+    const int tid = threadIdx.x;
     brt_setup(S, tcB, tcTw);
-    for (int e = tid; e < kTcG * 2 * kN; e += kTcThreads) (&S.acc[0][0][0])[e] = 0u;
-    // digits [g][r][1024] -> tile P / 4, row (P % 4)*32 + k2, K byte k1
-    for (int e = tid; e < kTcPolys * kN; e += kTcThreads) {
-        const int P = e / kN, c = e % kN, k1 = c >> 5, k2 = c & 31;
-        S.op[(P >> 2) * kOpTile + tc_off((P & 3) * 32 + k2, k1, kA1Lbo, kA1Sbo)] = (unsigned char)(digits[e] & 0xFF);
+    for (int e = tid; e < kTcLanes * 2 * kN; e += kTcThreads) {
+        const int L = e / (2 * kN);
+        (&S.grp[L / kTcG].acc[L % kTcG][0][0])[e % (2 * kN)] = 0u;
+    }
+    // digits [L][r][1024] -> group L / 2, tile P / 4 (P = (L % 2)*6 + r), row (P % 4)*32 + k2, K byte k1
+    for (int e = tid; e < kTcLanes * 6 * kN; e += kTcThreads) {
+        const int L = e / (6 * kN), r = (e / kN) % 6, c = e % kN, k1 = c >> 5, k2 = c & 31;
+        const int P = (L % kTcG) * 6 + r;
+        S.grp[L / kTcG].op[(P >> 2) * kOpTile + tc_off((P & 3) * 32 + k2, k1, kA1Lbo, kA1Sbo)] =
+            (unsigned char)(digits[e] & 0xFF);
     }
     fence_async_smem();
     __syncthreads();
-    uint32_t k = 0;
-    if (warp == kTcCompWarps) {
-        if ((tid & 31) == 0) {
-            uint32_t gph = 0, aph = 0;
-            brt_mma_step(S, k, gph, aph);
-        }
-        __syncwarp();
-    } else {
-        brt_comp_step(S, bk4, k);
-    }
+    brt_main<true>(S, bk4, 1);
     __syncthreads();
-    for (int e = tid; e < kTcG * 2 * kN; e += kTcThreads) res[e] = (&S.acc[0][0][0])[e];
+    for (int e = tid; e < kTcLanes * 2 * kN; e += kTcThreads) {
+        const int L = e / (2 * kN);
+        res[e] = (&S.grp[L / kTcG].acc[L % kTcG][0][0])[e % (2 * kN)];
+    }
     brt_teardown(S);
 }
 
@@ -475,7 +494,7 @@ static size_t brt_smem_bytes() { return sizeof(BrtSmem); }
 int launch_brt(const BrArgs& A, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw, cudaStream_t st) {
     static_assert(sizeof(BrtSmem) <= 232448, "brt shared memory");
     if (ensure_smem_attr<brt_kernel>(brt_smem_bytes())) return -1;
-    const int blocks = (A.nlanes + kTcG - 1) / kTcG;
+    const int blocks = (A.nlanes + kTcLanes - 1) / kTcLanes;
     if (blocks == 0) return 0;
     brt_kernel<<<blocks, kTcThreads, brt_smem_bytes(), st>>>(A, bk4, tcB, tcTw);
     return 0;
