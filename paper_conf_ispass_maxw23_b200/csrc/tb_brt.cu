@@ -172,23 +172,26 @@ __device__ __forceinline__ void brt_comp_step(BrtSmem& S, BrtGroup& G, uint32_t 
     __syncwarp();
     if (lane == 0) mbar_arrive(&G.gate);
     // ---- ep1: tile t, thread (P = 4t + qd, k2 = lane), j1 in this quad's half: C[j1][k2] -> A2 row (qd, j1)
+    uint2 twr[16];                                       // this thread's 16 forward twiddles (all tiles)
+#pragma unroll
+    for (int j = 0; j < 16; j++) twr[j] = S.twF[32 * (16 * hq + j) + lane];
     for (int t = 0; t < kTcTiles; t++) {
         const uint32_t kk = k + t, slot = kk % kTcSlots;
         mbar_wait(&G.full[slot], (kk / kTcSlots) & 1);
         tc_fence_after();
         unsigned char* base = G.op + t * kOpTile + opw(qd * 32 + 16 * hq, lane);
-        const uint2* tw = S.twF + 32 * 16 * hq + lane;
 #pragma unroll
-        for (int jc = 0; jc < 4; jc++) {
-            uint32_t v[16];
-            tc_ld16(tq + 128 * slot + 16 * jc, v);
+        for (int jc = 0; jc < 4; jc += 2) {
+            uint32_t v[2][16];
+            tc_ld16(tq + 128 * slot + 16 * jc, v[0]);
+            tc_ld16(tq + 128 * slot + 16 * jc + 16, v[1]);
             tc_wait_ld();
 #pragma unroll
-            for (int u = 0; u < 4; u++) {
+            for (int u = 0; u < 8; u++) {
                 const int j = 4 * jc + u;                  // j1 = 16 hq + j
-                const uint32_t x = limbs_s(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3]);
-                const uint2 w = tw[32 * j];
-                *reinterpret_cast<uint32_t*>(base + (j >> 3) * kOpSbo + (j & 7) * 16) = shoup_mul(x, w.x, w.y);
+                const uint32_t* y = &v[u >> 2][4 * (u & 3)];
+                const uint32_t x = limbs_s(y[0], y[1], y[2], y[3]);
+                *reinterpret_cast<uint32_t*>(base + (j >> 3) * kOpSbo + (j & 7) * 16) = shoup_mul(x, twr[j].x, twr[j].y);
             }
         }
         fence_async_smem();
@@ -207,34 +210,46 @@ __device__ __forceinline__ void brt_comp_step(BrtSmem& S, BrtGroup& G, uint32_t 
         tc_fence_after();
         unsigned char* base = G.op + t * kOpTile + opw(qd * 32 + lane, 16 * hq);
 #pragma unroll
-        for (int c = 0; c < 4; c++) {
-            uint32_t v[16];
-            tc_ld16(tq + 128 * slot + 16 * c, v);
+        for (int c = 0; c < 4; c += 2) {
+            uint32_t v[2][16];
+            tc_ld16(tq + 128 * slot + 16 * c, v[0]);
+            tc_ld16(tq + 128 * slot + 16 * c + 16, v[1]);
             tc_wait_ld();
-            uint4 o;
-            o.x = red_2p(limbs_u(v[0], v[1], v[2], v[3]));
-            o.y = red_2p(limbs_u(v[4], v[5], v[6], v[7]));
-            o.z = red_2p(limbs_u(v[8], v[9], v[10], v[11]));
-            o.w = red_2p(limbs_u(v[12], v[13], v[14], v[15]));
-            *reinterpret_cast<uint4*>(base + c * kOpLbo) = o;
+#pragma unroll
+            for (int h = 0; h < 2; h++) {
+                uint4 o;
+                o.x = red_2p(limbs_u(v[h][0], v[h][1], v[h][2], v[h][3]));
+                o.y = red_2p(limbs_u(v[h][4], v[h][5], v[h][6], v[h][7]));
+                o.z = red_2p(limbs_u(v[h][8], v[h][9], v[h][10], v[h][11]));
+                o.w = red_2p(limbs_u(v[h][12], v[h][13], v[h][14], v[h][15]));
+                *reinterpret_cast<uint4*>(base + (c + h) * kOpLbo) = o;
+            }
         }
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&G.empty[slot]);
     }
     k += kTcTiles;
-    grp_sync(grp);                                       // every ep2 tile of the group written
-    // ---- MAC: coefficient (j1, j2 = lane) of the 2 lanes, M_o = sum_r A_r BK4[r][o] (a4.3), in place per thread
+    // ---- MAC: coefficient (j1, j2 = lane) of the 2 lanes, M_o = sum_r A_r BK4[r][o] (a4.3), in place per thread.
+    // The first row's BK record is requested before the group barrier (its L2 latency overlaps the wait).
     {
         const uint32_t R = c_misc[0], Rp = c_misc[1];
         const uint32_t lanew = (lane >> 2) * kOpLbo + (lane & 3) * 4;
+        uint4 Bn[kBk4Rec / 4];
+        const uint4* rec0 = reinterpret_cast<const uint4*>(bk4 + (size_t)(gw * 32 + lane) * kBk4Rec);
+#pragma unroll
+        for (int q = 0; q < kBk4Rec / 4; q++) Bn[q] = __ldg(rec0 + q);
+        grp_sync(grp);                                   // every ep2 tile of the group written
         for (int j1 = gw; j1 < 32; j1 += kTcGWarps) {
-            const uint4* rec = reinterpret_cast<const uint4*>(bk4 + (size_t)(j1 * 32 + lane) * kBk4Rec);
             uint32_t B[kBk4Rec];
+            if (j1 != gw) {
+                const uint4* rec = reinterpret_cast<const uint4*>(bk4 + (size_t)(j1 * 32 + lane) * kBk4Rec);
+#pragma unroll
+                for (int q = 0; q < kBk4Rec / 4; q++) Bn[q] = __ldg(rec + q);
+            }
 #pragma unroll
             for (int q = 0; q < kBk4Rec / 4; q++) {
-                const uint4 b4 = __ldg(rec + q);
-                B[4 * q] = b4.x; B[4 * q + 1] = b4.y; B[4 * q + 2] = b4.z; B[4 * q + 3] = b4.w;
+                B[4 * q] = Bn[q].x; B[4 * q + 1] = Bn[q].y; B[4 * q + 2] = Bn[q].z; B[4 * q + 3] = Bn[q].w;
             }
             const uint32_t rowoff = (j1 >> 3) * kOpSbo + (j1 & 7) * 16 + lanew;
             uint32_t D[kTcG][6];
@@ -263,23 +278,25 @@ __device__ __forceinline__ void brt_comp_step(BrtSmem& S, BrtGroup& G, uint32_t 
     if (lane == 0) mbar_arrive(&G.gate);
     // ---- ep3: tile m, thread (quadrant qd = g*2 + q, j1 = lane), k2 in this quad's half: D[j1][k2] -> E -> A4
     // tile m row (qd, k2) word j1 (the tile GEMM3 just consumed)
+#pragma unroll
+    for (int j = 0; j < 16; j++) twr[j] = S.twI[32 * (16 * hq + j) + lane];
     for (int t = 0; t < kTcTiles; t++) {
         const uint32_t kk = k + t, slot = kk % kTcSlots;
         mbar_wait(&G.full[slot], (kk / kTcSlots) & 1);
         tc_fence_after();
         unsigned char* base = G.op + t * kOpTile + opw(qd * 32 + 16 * hq, lane);
-        const uint2* tw = S.twI + 32 * 16 * hq + lane;
 #pragma unroll
-        for (int c = 0; c < 4; c++) {
-            uint32_t v[16];
-            tc_ld16(tq + 128 * slot + 16 * c, v);
+        for (int c = 0; c < 4; c += 2) {
+            uint32_t v[2][16];
+            tc_ld16(tq + 128 * slot + 16 * c, v[0]);
+            tc_ld16(tq + 128 * slot + 16 * c + 16, v[1]);
             tc_wait_ld();
 #pragma unroll
-            for (int u = 0; u < 4; u++) {
+            for (int u = 0; u < 8; u++) {
                 const int j = 4 * c + u;                  // k2 = 16 hq + j
-                const uint32_t x = limbs_u(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3]);
-                const uint2 w = tw[32 * j];
-                *reinterpret_cast<uint32_t*>(base + (j >> 3) * kOpSbo + (j & 7) * 16) = shoup_mul(x, w.x, w.y);
+                const uint32_t* y = &v[u >> 2][4 * (u & 3)];
+                const uint32_t x = limbs_u(y[0], y[1], y[2], y[3]);
+                *reinterpret_cast<uint32_t*>(base + (j >> 3) * kOpSbo + (j & 7) * 16) = shoup_mul(x, twr[j].x, twr[j].y);
             }
         }
         fence_async_smem();
@@ -299,14 +316,16 @@ __device__ __forceinline__ void brt_comp_step(BrtSmem& S, BrtGroup& G, uint32_t 
         tc_fence_after();
         uint32_t* acc = &G.acc[qd >> 1][qd & 1][32 * 16 * hq + lane];
 #pragma unroll
-        for (int c = 0; c < 4; c++) {
-            uint32_t v[16];
-            tc_ld16(tq + 128 * slot + 16 * c, v);
+        for (int c = 0; c < 4; c += 2) {
+            uint32_t v[2][16];
+            tc_ld16(tq + 128 * slot + 16 * c, v[0]);
+            tc_ld16(tq + 128 * slot + 16 * c + 16, v[1]);
             tc_wait_ld();
 #pragma unroll
-            for (int u = 0; u < 4; u++) {
+            for (int u = 0; u < 8; u++) {
                 const int j = 4 * c + u;                  // k1 = 16 hq + j
-                const uint32_t a = lift_centred(red_2p(limbs_u(v[4 * u], v[4 * u + 1], v[4 * u + 2], v[4 * u + 3])));
+                const uint32_t* y = &v[u >> 2][4 * (u & 3)];
+                const uint32_t a = lift_centred(red_2p(limbs_u(y[0], y[1], y[2], y[3])));
                 acc[32 * j] += a << (11 * t);
             }
         }

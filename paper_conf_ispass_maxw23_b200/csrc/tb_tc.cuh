@@ -77,11 +77,13 @@ __device__ __forceinline__ void tc_ld16(uint32_t taddr, uint32_t (&v)[16]) {
 __device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
 }
+// try_wait with a suspend-time hint: a waiting thread sleeps in the barrier instead of re-issuing the test
+// (the spinning MMA thread otherwise takes issue slots from the compute warps of its sub-partition)
 __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
     asm volatile(
-        "{\n .reg .pred p;\n TCW_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "{\n .reg .pred p;\n TCW_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
         " @!p bra TCW_%=;\n}\n" ::"r"(smem_u32(b)),
-        "r"(parity)
+        "r"(parity), "r"(0x100000u)
         : "memory");
 }
 
