@@ -74,16 +74,22 @@ struct BrtSmem {
 constexpr uint32_t kW16p = (uint32_t)((((uint64_t)1 << 48)) / kP);    // Shoup companion of 2^16
 // operands < 2p (top byte <= 127): Y0 + 2^8 Y1 <= 32 (3*255 + 127) 255 * 257 < 1.9e9, hi 2^16 mod p < 2p,
 // so the sum stays below 4.1e9 < 4p: no reduction of the low half is needed
+// The shift-adds are written as funnel shifts (SHF) and three-input adds (IADD3) so that ptxas keeps them on the
+// ALU pipe: plain `y0 + (y1 << 8)` becomes an IMAD on the FMA-heavy pipe, which the Shoup products and the MAC
+// already load (measured: IMAD was 28 % of the kernel's executed instructions).
+__device__ __forceinline__ uint32_t shl_alu(uint32_t x, int s) { return __funnelshift_l(0u, x, s); }
 __device__ __forceinline__ uint32_t limbs_u(uint32_t y0, uint32_t y1, uint32_t y2, uint32_t y3) {
-    const uint32_t lo = y0 + (y1 << 8), hi = y2 + (y3 << 8);
+    const uint32_t hi = y2 + shl_alu(y3, 8) + c_zero;
     const uint32_t q = __umulhi(hi, kW16p);
-    return lo + ((hi << 16) - q * kP);
+    const uint32_t r = shl_alu(hi, 16) - q * kP;                   // hi 2^16 mod p in [0, 2p)
+    return y0 + shl_alu(y1, 8) + r;
 }
 // signed limbs (s8 digits x u8, |Y_b| < 2^19): lo + p, hi + p are in (0, 2p); result < 4p
 __device__ __forceinline__ uint32_t limbs_s(uint32_t y0, uint32_t y1, uint32_t y2, uint32_t y3) {
-    const uint32_t lo = y0 + (y1 << 8) + kP, hi = y2 + (y3 << 8) + kP;
+    const uint32_t hi = y2 + shl_alu(y3, 8) + kP;
     const uint32_t q = __umulhi(hi, kW16p);
-    return lo + ((hi << 16) - q * kP);
+    const uint32_t r = shl_alu(hi, 16) - q * kP;
+    return y0 + shl_alu(y1, 8) + (r + kP + c_zero);
 }
 __device__ __forceinline__ void mbar_arrive(uint64_t* b) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
