@@ -152,11 +152,16 @@ int tb_ipc_close(tb_ctx* ctx, void* base);
 int tb_run_netlist(tb_ctx* ctx, const tb_dev_netlist* dnet, uint32_t* wires, int64_t stride, tb_stream stream);
 
 /* End-to-end netlist evaluation through HOST buffers: copies the n_inputs input ciphertexts (rows of
- * in_stride words, host) into a context-owned device wire array, runs every level, gathers the rows of
- * the n_outputs wires listed in output_wires (original wire ids, host array) and copies them to
- * host_outputs (rows of out_stride >= 631 words).  Synchronous. */
+ * in_stride words, host) into a context-owned device wire array, runs every level, and copies the rows of
+ * the n_outputs wires listed in output_wires (original wire ids, host array) to host_outputs (rows of
+ * out_stride >= 631 words).  The input copies run on their own stream in the order of the level that first reads
+ * them (level L waits only for its inputs) and the outputs of level L are copied back while level L + 1 runs
+ * (SURVEY 8(f) f1); pinned host buffers make the copies asynchronous.  Synchronous. */
 int tb_run_netlist_host(tb_ctx* ctx, const tb_dev_netlist* dnet, const uint32_t* host_inputs, int64_t in_stride,
                         const int64_t* output_wires, int64_t n_outputs, uint32_t* host_outputs, int64_t out_stride);
+/* tb_run_netlist_host: overlap the copies with the level loop (1, default) or run copy, levels, copy back one
+ * after the other (0) -- for measuring the overlap. */
+int tb_set_host_overlap(tb_ctx* ctx, int enable);
 
 /* ---- per-kernel timing (CUDA events recorded around every launch on the launching stream) ---------- */
 /* enable != 0 starts recording (and clears previous records); 0 stops. */
@@ -206,6 +211,23 @@ int tb_set_narrow_kernel(tb_ctx* ctx, int kernel);
  * fit on the device, 32 on B200), 0 = Algorithm 1 as is.  Output bytes are identical either way (each gate's
  * result depends only on its inputs).  Affects netlists uploaded afterwards.  lanes < -1: TB_EINVAL. */
 int tb_set_level_capacity(tb_ctx* ctx, int64_t lanes);
+/* Level order of netlists uploaded afterwards, for a level loop over `world` ranks (P:263's
+ * dependency-driven batching carried across GPUs): every level is cut into `world` contiguous chunks of
+ * ceil(n / world) gates (rank r evaluates chunk r), and each chunk begins with the gates whose inputs from the
+ * previous level were all produced by the same rank -- those can run before the previous level's exchange
+ * barrier.  Output bytes do not depend on the order.  Default 1 (ascending gate index).  world < 1: TB_EINVAL. */
+int tb_set_plan_world(tb_ctx* ctx, int world);
+/* Host-only plan of tb_netlist_upload for `world` ranks and capacity `lanes` (0 = Algorithm 1): level offsets
+ * [n_levels + 1], row of every wire, and early[(level - 1) * world + rank] (see tb_netlist_early).  Call with
+ * null arrays to get n_levels first.  Bad arguments: TB_EINVAL. */
+int tb_netlist_plan_world(const tb_netlist* net, int64_t lanes, int world, int64_t* n_levels, int64_t* level_off,
+                          int64_t* row_of_wire, int64_t* early);
+/* The world size a device netlist was planned for (tb_set_plan_world at upload time). */
+int tb_netlist_world(const tb_dev_netlist* dnet, int* world);
+/* Number of "early" gates at the start of rank `rank`'s chunk of `level` (1-based): gates whose inputs are in
+ * levels < level - 1 or in the same rank's chunk of level - 1, so rank `rank` can evaluate them right after its
+ * own part of level - 1, before that level's exchange.  Level 1: the whole chunk.  Out of range: TB_EINVAL. */
+int tb_netlist_early(const tb_dev_netlist* dnet, int64_t level, int rank, int64_t* n_early);
 /* Gates per key-switch CTA (8, 16 or 32; default 8): each tile streams the 62 MB KSK once from L2. */
 int tb_set_ks_tile(tb_ctx* ctx, int gates);
 /* Device bytes a context holds for keys (BK NTT + KSK). */

@@ -79,6 +79,18 @@ class DevNetlist:
             v = [ctypes.c_int64() for _ in range(4)]
             _native.check(_native.lib().tb_netlist_level(h, L, *[ctypes.byref(x) for x in v]))
             self.levels.append(tuple(int(x.value) for x in v))
+        w = ctypes.c_int()
+        _native.check(_native.lib().tb_netlist_world(h, ctypes.byref(w)))
+        self.world = int(w.value)     # ranks the level order was planned for (tb_set_plan_world)
+
+    def early(self, rank: int):
+        """per level, this rank's early-gate count (tb_netlist_early); needs world == the loop's world size"""
+        out = []
+        for L in range(1, self.n_levels + 1):
+            e = ctypes.c_int64()
+            _native.check(_native.lib().tb_netlist_early(self._h, L, rank, ctypes.byref(e)))
+            out.append(int(e.value))
+        return out
 
     @property
     def n_boot(self) -> int:
@@ -252,8 +264,14 @@ class Context:
         return int(v.value)
 
     # ---- netlists (Algorithm 1) ----
-    def upload(self, net: Netlist) -> DevNetlist:
-        return DevNetlist(self, net)
+    def upload(self, net: Netlist, world: int = 1) -> DevNetlist:
+        """Levelise and upload; world > 1 orders every level for a loop over that many ranks so each rank's chunk
+        starts with the gates it can run before the previous level's exchange (tb_set_plan_world)."""
+        _native.check(_native.lib().tb_set_plan_world(self._h, world))
+        try:
+            return DevNetlist(self, net)
+        finally:
+            _native.lib().tb_set_plan_world(self._h, 1)
 
     def wire_array(self, dnet: DevNetlist, slack_rows: int = 0, stride: int = WIRE_STRIDE) -> torch.Tensor:
         return torch.zeros((dnet.n_rows + slack_rows, stride), dtype=torch.int32, device=self.device)
@@ -263,12 +281,15 @@ class Context:
         _native.check(_native.lib().tb_run_level(self._h, dnet._h, level, g0, g1, _ptr(wires), wires.stride(0),
                                                  _stream_handle(stream)))
 
-    def run_netlist(self, dnet: DevNetlist, wires: torch.Tensor, group=None, stream=None, exchange: str = "fused"):
+    def run_netlist(self, dnet: DevNetlist, wires: torch.Tensor, group=None, stream=None, exchange: str = "fused",
+                    early_start: bool = True):
         """Evaluate every level.  Without a process group: one device (tb_run_netlist).  With one: each
         level's gates are split into R contiguous chunks and rank r evaluates chunk r; the level's output rows
         reach every rank either through the key-switch kernels' own stores into the peers' wire arrays
         (exchange="fused": CUDA-IPC peer memory, tb_set_peer_wires, then a barrier) or through an in-place
-        all-gather over the process group (exchange="allgather").  DESIGN.md "Multi-GPU"."""
+        all-gather over the process group (exchange="allgather").  If dnet was uploaded for this world size
+        (upload(net, world=R)) and the exchange is fused, each rank starts the next level's locally ready gates
+        before the current level's barrier (early_start).  DESIGN.md "Multi-GPU"."""
         _check_dev(wires, self.device, "wires")
         if group is None:
             _native.check(_native.lib().tb_run_netlist(self._h, dnet._h, _ptr(wires), wires.stride(0),
@@ -282,8 +303,11 @@ class Context:
             self.attach_peers(wires, group)
         # the per-level barrier / all-gather must be ordered on the stream the level kernels run on: make it the
         # current stream for the loop (collectives order against torch's current stream)
+        import torch.distributed as dist
+        R, r = dist.get_world_size(group), dist.get_rank(group)
+        early = dnet.early(r) if (dnet.world == R and R > 1 and early_start) else None
         with torch.cuda.stream(stream) if stream is not None else _nullcontext():
-            parallel.level_loop(levels, wires, run, group, fused=exchange == "fused")
+            parallel.level_loop(levels, wires, run, group, fused=exchange == "fused", early=early)
 
     # ---- fused all-gather: the other ranks' wire arrays mapped into this process (CUDA IPC) ----
     def attach_peers(self, wires: torch.Tensor, group):
@@ -345,6 +369,10 @@ class Context:
             for b in bases:
                 _native.lib().tb_ipc_close(self._h, ctypes.c_void_p(b))
         self._peer_bases, self._peer_key = [], None
+
+    def set_host_overlap(self, enable: bool):
+        """run_netlist_host*: overlap the host copies with the level loop (default) or serialise them"""
+        _native.check(_native.lib().tb_set_host_overlap(self._h, 1 if enable else 0))
 
     def run_netlist_host(self, dnet: DevNetlist, inputs: np.ndarray, output_wires) -> np.ndarray:
         """End-to-end through HOST buffers (tb_run_netlist_host): input ciphertexts [n_inputs, >=631] u32 ->

@@ -104,6 +104,11 @@ SIGNATURES = {
     "tb_tc_mma_test": (ctypes.c_int, [_vp, _vp, _vp, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                       ctypes.c_int, _vp]),
     "tb_tc_muladd": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
+    "tb_set_plan_world": (ctypes.c_int, [_vp, ctypes.c_int]),
+    "tb_netlist_world": (ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_int)]),
+    "tb_netlist_early": (ctypes.c_int, [_vp, _i64, ctypes.c_int, ctypes.POINTER(_i64)]),
+    "tb_netlist_plan_world": (ctypes.c_int, [_vp, _i64, ctypes.c_int, ctypes.POINTER(_i64), _vp, _vp, _vp]),
+    "tb_set_host_overlap": (ctypes.c_int, [_vp, ctypes.c_int]),
     "tb_microbench": (ctypes.c_int, [_vp, ctypes.c_int, ctypes.POINTER(ctypes.c_double),
                                      ctypes.POINTER(ctypes.c_double)]),
     "tb_last_error": (ctypes.c_char_p, []),

@@ -77,10 +77,6 @@ int run_tc_mma_test(const uint8_t* A, const uint8_t* B, int K, int N, int a_sign
 
 }  // namespace tb
 
-namespace tb {
-void launch_gather_rows(const uint32_t* src, int64_t stride, const int64_t* rows, int64_t n, uint32_t* out,
-                        cudaStream_t st);
-}  // namespace tb
 
 namespace tb {
 int set_fft_constants(const double2* zeta16);

@@ -240,18 +240,3 @@ void launch_ksk_relayout(const uint32_t* src, uint32_t* dst, cudaStream_t st) {
 }
 
 }  // namespace tb
-
-namespace tb {
-// out[k] = src[rows[k]] (631 words per row, `stride`-word rows): output gather of tb_run_netlist_host
-__global__ void gather_rows_kernel(const uint32_t* src, int64_t stride, const int64_t* rows, int64_t n, uint32_t* out) {
-    const int64_t k = blockIdx.x;
-    if (k >= n) return;
-    const uint32_t* s = src + rows[k] * stride;
-    uint32_t* d = out + k * stride;
-    for (int w = threadIdx.x; w <= kn; w += blockDim.x) d[w] = s[w];
-}
-void launch_gather_rows(const uint32_t* src, int64_t stride, const int64_t* rows, int64_t n, uint32_t* out,
-                        cudaStream_t st) {
-    if (n > 0) gather_rows_kernel<<<(unsigned)n, 128, 0, st>>>(src, stride, rows, n, out);
-}
-}  // namespace tb

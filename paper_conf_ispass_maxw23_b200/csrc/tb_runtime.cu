@@ -68,9 +68,13 @@ struct tb_ctx {
                                             // 11 = brl (4-SM cluster per lane, FP64 path), 0 = auto:
                                             // brl while the lanes fit in one wave of its clusters, else br9
     int brl_wave = -2;                      // co-resident brl clusters (queried on first use)
+    int plan_world = 1;                     // netlist upload: order each level for this many ranks (early gates first)
     int64_t level_capacity = -1;            // netlist upload: re-levelise to <= this many lanes per level where
                                             // slack allows (0 = Algorithm 1 as is, -1 = auto: brl_wave)
     cudaStream_t own = nullptr;             // internal stream for load / host-buffer calls
+    cudaStream_t h2d = nullptr, d2h = nullptr;   // tb_run_netlist_host copy streams (overlap with the levels)
+    std::vector<cudaEvent_t> hev;           // tb_run_netlist_host events (per level: inputs landed, outputs ready)
+    int overlap_host = 1;                   // tb_run_netlist_host: overlap copies with the level loop
     uint2* twF = nullptr;                   // [31][32]
     uint2* twI = nullptr;
     double2* fftB = nullptr;                // FP64 FFT per-lane twiddles: stages 5-8 [15][32], stage 9 [8][32]
@@ -95,8 +99,6 @@ struct tb_ctx {
     size_t stage_words = 0;
     uint32_t* hwires = nullptr;             // tb_run_netlist_host device wire array
     size_t hwires_words = 0;
-    int64_t* hidx = nullptr;                // tb_run_netlist_host gather rows
-    int64_t hidx_n = 0;
     uint32_t** peers = nullptr;             // fused all-gather: device array of the other ranks' wire bases
     int32_t npeers = 0;
     const uint32_t* peer_own = nullptr;     // the local wire array the peers mirror (other arrays: no peer stores)
@@ -137,6 +139,10 @@ struct tb_dev_netlist {
     std::vector<int64_t> lane_off;          // [n_gates + 1] lane prefix over level-sorted gates
     std::vector<int64_t> boot_prefix;       // [n_gates + 1] bootstrapped gates (non-NOT) prefix
     std::vector<int64_t> row_of_wire;       // [n_inputs + n_gates]
+    int world = 1;                          // ranks the level order was planned for
+    std::vector<int64_t> in_level;          // [n_inputs] first level that reads the input (n_levels + 1: none)
+    std::vector<int64_t> early;             // [n_levels][world]: gates at the start of rank r's chunk of a level
+                                            // whose inputs are local once r has run its part of the level before
     LaneDesc* ldesc = nullptr;
     GateDesc* gdesc = nullptr;
 };
@@ -297,11 +303,13 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
     cudaFree(c->gdesc);
     cudaFree(c->stage);
     cudaFree(c->hwires);
-    cudaFree(c->hidx);
     cudaFree(c->ks_scratch);
     cudaFree(c->peers);
     for (cudaEvent_t e : c->ev_pool) cudaEventDestroy(e);
     if (c->own) cudaStreamDestroy(c->own);
+    if (c->h2d) cudaStreamDestroy(c->h2d);
+    if (c->d2h) cudaStreamDestroy(c->d2h);
+    for (cudaEvent_t e : c->hev) cudaEventDestroy(e);
     delete c;
     return TB_OK;
 }
@@ -358,6 +366,26 @@ extern "C" int tb_set_level_capacity(tb_ctx* c, int64_t lanes) {
 extern "C" int tb_set_narrow_lanes(tb_ctx* c, int64_t lanes) {
     if (!c || lanes < 0) return fail(TB_EINVAL, "narrow-level threshold must be >= 0");
     c->narrow_lanes = lanes;
+    return TB_OK;
+}
+
+extern "C" int tb_set_plan_world(tb_ctx* c, int world) {
+    if (!c || world < 1 || world > 1024) return fail(TB_EINVAL, "world size must be 1..1024");
+    c->plan_world = world;
+    return TB_OK;
+}
+
+extern "C" int tb_netlist_early(const tb_dev_netlist* d, int64_t level, int rank, int64_t* n_early) {
+    if (!d || !n_early) return fail(TB_EINVAL, "null argument");
+    if (level < 1 || level > d->n_levels) return fail(TB_EINVAL, "level out of range");
+    if (rank < 0 || rank >= d->world) return fail(TB_EINVAL, "rank outside the world size the netlist was planned for");
+    *n_early = d->early[(size_t)(level - 1) * d->world + rank];
+    return TB_OK;
+}
+
+extern "C" int tb_netlist_world(const tb_dev_netlist* d, int* world) {
+    if (!d || !world) return fail(TB_EINVAL, "null argument");
+    *world = d->world;
     return TB_OK;
 }
 
@@ -791,8 +819,75 @@ static void relevel_capacity(const tb_netlist* net, std::vector<int64_t>& lv, in
 // [0, n_inputs); the gates of level L follow those of level L-1, ascending original index inside a level.
 // level_off (0-based, n_levels + 1 entries) are gate offsets into that order; order[k] = original gate index
 // of the k-th gate.
+// Level order for R ranks (start a rank's locally ready gates before the level barrier).  Each
+// level is cut into R contiguous chunks (parallel.shard: ceil(n / R) gates each).  A gate of level L is "early"
+// for rank r if every input it reads from level L - 1 lies in r's chunk of level L - 1 (inputs of older levels
+// were exchanged at earlier barriers).  Rank r's chunk of level L is filled with the gates that are early for r
+// (affinity r, then gates with no level-(L-1) input), then with the rest; its early gates come first, so they
+// are a prefix [g0, g0 + early) that r can run before the barrier of level L - 1.  Outputs do not depend on the
+// order (each gate's result depends only on its input bytes); R = 1 keeps ascending original indices.
+static void order_for_world(const tb_netlist* net, const std::vector<int64_t>& lv, int64_t nlev,
+                            const std::vector<int64_t>& level_off, std::vector<int64_t>& order, int world,
+                            std::vector<int64_t>& early) {
+    const int64_t ni = net->n_inputs;
+    early.assign((size_t)nlev * world, 0);
+    std::vector<int64_t> rank_of_gate((size_t)net->n_gates, -1);   // rank owning the gate in its level
+    auto ins = [&](int64_t g, int k) -> int64_t {
+        const int t = net->type[g];
+        if (k == 0) return net->in0[g];
+        if (k == 1) return t == TB_NOT ? -1 : net->in1[g];
+        return t == TB_MUX ? net->in2[g] : -1;
+    };
+    for (int64_t L = 1; L <= nlev; L++) {
+        const int64_t a = level_off[L - 1], n = level_off[L] - a;
+        const int64_t chunk = (n + world - 1) / world;
+        // affinity: -1 = no input from level L - 1 ("free"), r = all such inputs on rank r, -2 = several ranks
+        std::vector<std::vector<int64_t>> aff((size_t)world);
+        std::vector<int64_t> freeg, mixed;
+        for (int64_t k = 0; k < n; k++) {
+            const int64_t g = order[a + k];
+            int64_t r = -1;
+            for (int q = 0; q < 3; q++) {
+                const int64_t w = ins(g, q);
+                if (w < ni || lv[w - ni] != L - 1) continue;
+                const int64_t rw = rank_of_gate[w - ni];
+                r = (r == -1 || r == rw) ? rw : -2;
+            }
+            if (r == -1) freeg.push_back(g);
+            else if (r == -2) mixed.push_back(g);
+            else aff[(size_t)r].push_back(g);
+        }
+        std::vector<std::vector<int64_t>> part((size_t)world);
+        std::vector<int64_t> rest, cap((size_t)world);
+        for (int r = 0; r < world; r++) {
+            cap[r] = std::max<int64_t>(0, std::min<int64_t>((r + 1) * chunk, n) - std::min<int64_t>(r * chunk, n));
+            for (int64_t g : aff[r]) {
+                if ((int64_t)part[r].size() < cap[r]) part[r].push_back(g);
+                else rest.push_back(g);
+            }
+        }
+        size_t fi = 0;
+        for (int r = 0; r < world; r++)
+            while ((int64_t)part[r].size() < cap[r] && fi < freeg.size()) part[r].push_back(freeg[fi++]);
+        for (int r = 0; r < world; r++) early[(size_t)(L - 1) * world + r] = (int64_t)part[r].size();
+        for (; fi < freeg.size(); fi++) rest.push_back(freeg[fi]);
+        rest.insert(rest.end(), mixed.begin(), mixed.end());
+        std::sort(rest.begin(), rest.end());
+        size_t ri = 0;
+        int64_t k = a;
+        for (int r = 0; r < world; r++) {
+            while ((int64_t)part[r].size() < cap[r] && ri < rest.size()) part[r].push_back(rest[ri++]);
+            for (int64_t g : part[r]) {
+                order[k++] = g;
+                rank_of_gate[g] = r;
+            }
+        }
+    }
+}
+
 static int plan_impl(const tb_netlist* net, int64_t* n_levels, std::vector<int64_t>& level_off,
-                     std::vector<int64_t>& order, std::vector<int64_t>& row_of_wire, int64_t cap = 0) {
+                     std::vector<int64_t>& order, std::vector<int64_t>& row_of_wire, int64_t cap = 0,
+                     int world = 1, std::vector<int64_t>* early = nullptr) {
     std::vector<int64_t> lv;
     int64_t nlev = 0;
     int rc = levelise_impl(net, lv, &nlev);
@@ -806,6 +901,14 @@ static int plan_impl(const tb_netlist* net, int64_t* n_levels, std::vector<int64
     std::vector<int64_t> pos(level_off.begin(), level_off.end());
     order.assign((size_t)ng, 0);
     for (int64_t g = 0; g < ng; g++) order[pos[lv[g] - 1]++] = g;
+    if (early) {
+        if (world > 1) {
+            order_for_world(net, lv, nlev, level_off, order, world, *early);
+        } else {
+            early->assign((size_t)nlev, 0);
+            for (int64_t L = 1; L <= nlev; L++) (*early)[L - 1] = L == 1 ? level_off[1] : 0;
+        }
+    }
     row_of_wire.resize((size_t)(ni + ng));
     for (int64_t w = 0; w < ni; w++) row_of_wire[w] = w;
     for (int64_t k = 0; k < ng; k++) row_of_wire[ni + order[k]] = ni + k;
@@ -829,6 +932,19 @@ extern "C" int tb_netlist_plan_capacity(const tb_netlist* net, int64_t lanes, in
     return TB_OK;
 }
 
+extern "C" int tb_netlist_plan_world(const tb_netlist* net, int64_t lanes, int world, int64_t* n_levels,
+                                     int64_t* level_off, int64_t* row_of_wire, int64_t* early) {
+    if (!net || !n_levels) return fail(TB_EINVAL, "null argument");
+    if (lanes < 0 || world < 1 || world > 1024) return fail(TB_EINVAL, "capacity must be >= 0, world 1..1024");
+    std::vector<int64_t> lo, order, rows, ea;
+    int rc = plan_impl(net, n_levels, lo, order, rows, lanes, world, &ea);
+    if (rc) return rc;
+    if (level_off) std::copy(lo.begin(), lo.end(), level_off);
+    if (row_of_wire) std::copy(rows.begin(), rows.end(), row_of_wire);
+    if (early) std::copy(ea.begin(), ea.end(), early);
+    return TB_OK;
+}
+
 extern "C" int tb_netlist_upload(tb_ctx* c, const tb_netlist* net, tb_dev_netlist** out) {
     if (!c || !net || !out) return fail(TB_EINVAL, "null argument");
     *out = nullptr;
@@ -841,13 +957,23 @@ extern "C" int tb_netlist_upload(tb_ctx* c, const tb_netlist* net, tb_dev_netlis
         if (c->brl_wave == -2) c->brl_wave = brl_wave_lanes();
         cap = c->brl_wave > 0 ? c->brl_wave : 0;
     }
-    int rc = plan_impl(net, &d->n_levels, d->level_off, order, d->row_of_wire, cap);
+    d->world = c->plan_world;
+    int rc = plan_impl(net, &d->n_levels, d->level_off, order, d->row_of_wire, cap, d->world, &d->early);
     if (rc) {
         delete d;
         return rc;
     }
     const int64_t ni = net->n_inputs, ng = net->n_gates;
     d->n_inputs = ni; d->n_gates = ng;
+    d->in_level.assign((size_t)ni, d->n_levels + 1);
+    for (int64_t L = 1; L <= d->n_levels; L++)
+        for (int64_t k = d->level_off[L - 1]; k < d->level_off[L]; k++) {
+            const int64_t g = order[k];
+            const int t = net->type[g];
+            const int64_t w[3] = {net->in0[g], t == TB_NOT ? -1 : net->in1[g], t == TB_MUX ? net->in2[g] : -1};
+            for (int64_t x : w)
+                if (x >= 0 && x < ni) d->in_level[x] = std::min(d->in_level[x], L);
+        }
     // descriptors in level-sorted order
     std::vector<GateDesc> gd((size_t)ng);
     std::vector<LaneDesc> ld;
@@ -1067,23 +1193,31 @@ extern "C" int tb_profile_read(tb_ctx* c, double* br_ms, int64_t* br_n, double* 
 }
 
 // ------------------------------------------------------------------------------------------ e2e host path
+extern "C" int tb_set_host_overlap(tb_ctx* c, int enable) {
+    if (!c) return fail(TB_EINVAL, "null context");
+    c->overlap_host = enable != 0;
+    return TB_OK;
+}
+
+// End to end through host buffers (the host side of one batch overlaps the device
+// work of another).  The input rows are copied on their own stream in the order of the level that first reads
+// them, and level L waits only for the inputs it reads; the requested outputs produced by level L are copied back
+// on a second stream while level L + 1 runs.  With overlap off (tb_set_host_overlap(0)) everything is serial.
 extern "C" int tb_run_netlist_host(tb_ctx* c, const tb_dev_netlist* d, const uint32_t* hin, int64_t in_stride,
                                    const int64_t* outw, int64_t n_out, uint32_t* hout, int64_t out_stride) {
     int rc = check_ready(c);
     if (rc) return rc;
     if (!d || (d->n_inputs > 0 && !hin) || (n_out > 0 && (!outw || !hout))) return fail(TB_EINVAL, "null argument");
     if (in_stride < kn + 1 || out_stride < kn + 1 || n_out < 0) return fail(TB_EINVAL, "bad stride or count");
-    const int64_t nw = d->n_inputs + d->n_gates;
+    const int64_t nw = d->n_inputs + d->n_gates, nL = d->n_levels;
     std::vector<int64_t> rows((size_t)n_out);
-    bool contiguous = true;
     for (int64_t k = 0; k < n_out; k++) {
         if (outw[k] < 0 || outw[k] >= nw) return fail(TB_EINVAL, "output wire out of range");
         rows[k] = d->row_of_wire[outw[k]];
-        if (k && rows[k] != rows[k - 1] + 1) contiguous = false;
     }
     TB_CUDA(cudaSetDevice(c->device));
     const int64_t S = kKsRow;                        // 632-word device rows
-    const size_t words = (size_t)(nw + std::max<int64_t>(n_out, 1)) * S;
+    const size_t words = (size_t)nw * S + 1;
     if (c->hwires_words < words) {
         cudaFree(c->hwires);
         c->hwires = nullptr;
@@ -1094,33 +1228,79 @@ extern "C" int tb_run_netlist_host(tb_ctx* c, const tb_dev_netlist* d, const uin
         }
         c->hwires_words = words;
     }
-    uint32_t* gather = c->hwires + (size_t)nw * S;
-    if (d->n_inputs > 0)
-        TB_CUDA(cudaMemcpy2DAsync(c->hwires, S * 4, hin, in_stride * 4, (kn + 1) * 4, d->n_inputs,
-                                  cudaMemcpyHostToDevice, c->own));
-    rc = tb_run_netlist(c, d, c->hwires, S, (tb_stream)c->own);
-    if (rc) return rc;
-    if (n_out > 0) {
-        const uint32_t* src = c->hwires + (size_t)rows[0] * S;
-        if (!contiguous) {
-            if (c->hidx_n < n_out) {
-                cudaFree(c->hidx);
-                c->hidx = nullptr;
-                c->hidx_n = 0;
-                if (cudaMalloc(&c->hidx, n_out * 8) != cudaSuccess) {
-                    cudaGetLastError();
-                    return fail(TB_ENOMEM, "index allocation failed");
-                }
-                c->hidx_n = n_out;
-            }
-            TB_CUDA(cudaMemcpyAsync(c->hidx, rows.data(), n_out * 8, cudaMemcpyHostToDevice, c->own));
-            launch_gather_rows(c->hwires, S, c->hidx, n_out, gather, c->own);
-            TB_CUDA(cudaGetLastError());
-            src = gather;
-        }
-        TB_CUDA(cudaMemcpy2DAsync(hout, out_stride * 4, src, S * 4, (kn + 1) * 4, n_out, cudaMemcpyDeviceToHost,
-                                  c->own));
+    const bool ov = c->overlap_host != 0;
+    if (ov && !c->h2d) TB_CUDA(cudaStreamCreateWithFlags(&c->h2d, cudaStreamNonBlocking));
+    if (ov && !c->d2h) TB_CUDA(cudaStreamCreateWithFlags(&c->d2h, cudaStreamNonBlocking));
+    cudaStream_t cs = c->own, hs = ov ? c->h2d : c->own, ds = ov ? c->d2h : c->own;
+    const size_t nev = 2 * (size_t)(nL + 2);
+    while (c->hev.size() < nev) {
+        cudaEvent_t e;
+        TB_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        c->hev.push_back(e);
     }
-    TB_CUDA(cudaStreamSynchronize(c->own));
+    auto ev_in = [&](int64_t L) { return c->hev[(size_t)L]; };             // inputs of level L landed
+    auto ev_out = [&](int64_t L) { return c->hev[(size_t)(nL + 2 + L)]; }; // level L's outputs are final
+    // ---- inputs: runs of consecutive rows with the same first level, in level order
+    std::vector<int64_t> by_level;                    // input rows sorted by (first level, row)
+    by_level.resize((size_t)d->n_inputs);
+    for (int64_t w = 0; w < d->n_inputs; w++) by_level[w] = w;
+    std::stable_sort(by_level.begin(), by_level.end(),
+                     [&](int64_t x, int64_t y) { return d->in_level[x] < d->in_level[y]; });
+    std::vector<char> has_in((size_t)nL + 2, 0);
+    for (size_t a = 0; a < by_level.size();) {
+        const int64_t L = d->in_level[by_level[a]];
+        size_t b = a + 1;
+        while (b < by_level.size() && d->in_level[by_level[b]] == L && by_level[b] == by_level[b - 1] + 1) b++;
+        TB_CUDA(cudaMemcpy2DAsync(c->hwires + (size_t)by_level[a] * S, S * 4, hin + (size_t)by_level[a] * in_stride,
+                                  in_stride * 4, (kn + 1) * 4, b - a, cudaMemcpyHostToDevice, hs));
+        const bool last_of_level = b == by_level.size() || d->in_level[by_level[b]] != L;
+        if (last_of_level) {
+            TB_CUDA(cudaEventRecord(ev_in(std::min(L, nL + 1)), hs));
+            has_in[(size_t)std::min(L, nL + 1)] = 1;
+        }
+        a = b;
+    }
+    // ---- outputs grouped by the level that produces them (0: an input passed through)
+    std::vector<int64_t> lvl_of_row;                  // level of a gate row
+    std::vector<std::vector<int64_t>> outs_at((size_t)nL + 1);
+    for (int64_t k = 0; k < n_out; k++) {
+        const int64_t r = rows[k];
+        int64_t L = 0;
+        if (r >= d->n_inputs)
+            L = (int64_t)(std::upper_bound(d->level_off.begin(), d->level_off.end(), r - d->n_inputs) -
+                          d->level_off.begin());
+        outs_at[(size_t)L].push_back(k);
+    }
+    auto copy_outs = [&](int64_t L) -> int {
+        const auto& ks = outs_at[(size_t)L];
+        for (size_t a = 0; a < ks.size();) {
+            size_t b = a + 1;
+            while (b < ks.size() && ks[b] == ks[b - 1] + 1 && rows[ks[b]] == rows[ks[b - 1]] + 1) b++;
+            TB_CUDA(cudaMemcpy2DAsync(hout + (size_t)ks[a] * out_stride, out_stride * 4,
+                                      c->hwires + (size_t)rows[ks[a]] * S, S * 4, (kn + 1) * 4, b - a,
+                                      cudaMemcpyDeviceToHost, ds));
+            a = b;
+        }
+        return TB_OK;
+    };
+    // ---- the level loop on the compute stream
+    for (int64_t L = 1; L <= nL; L++) {
+        if (has_in[(size_t)L]) TB_CUDA(cudaStreamWaitEvent(cs, ev_in(L), 0));
+        const int64_t n = d->level_off[L] - d->level_off[L - 1];
+        if ((rc = tb_run_level(c, d, L, 0, n, c->hwires, S, (tb_stream)cs))) return rc;
+        if (!outs_at[(size_t)L].empty()) {
+            TB_CUDA(cudaEventRecord(ev_out(L), cs));
+            TB_CUDA(cudaStreamWaitEvent(ds, ev_out(L), 0));
+            if ((rc = copy_outs(L))) return rc;
+        }
+    }
+    if (!outs_at[0].empty()) {                        // outputs that are inputs: after every input copy
+        for (int64_t L = 1; L <= nL + 1; L++)
+            if (has_in[(size_t)L]) TB_CUDA(cudaStreamWaitEvent(ds, ev_in(L), 0));
+        if ((rc = copy_outs(0))) return rc;
+    }
+    TB_CUDA(cudaStreamSynchronize(hs));
+    TB_CUDA(cudaStreamSynchronize(cs));
+    TB_CUDA(cudaStreamSynchronize(ds));
     return TB_OK;
 }

@@ -77,6 +77,23 @@ class Netlist:
         levels = [(self.n_inputs + int(off[L]), int(off[L + 1] - off[L])) for L in range(int(nl.value))]
         return levels, rows
 
+    def plan_world(self, world: int, capacity: int = 0):
+        """Host-only plan for a level loop over `world` ranks (tb_netlist_plan_world): (levels, row_of_wire, early)
+        with early[L - 1][r] = the gates at the start of rank r's chunk of level L that r can run before the
+        exchange of level L - 1."""
+        s = self.c_struct()
+        nl = ctypes.c_int64(0)
+        f = _native.lib().tb_netlist_plan_world
+        _native.check(f(ctypes.byref(s), capacity, world, ctypes.byref(nl), None, None, None))
+        L = int(nl.value)
+        off = np.zeros(L + 1, np.int64)
+        rows = np.zeros(self.n_wires, np.int64)
+        early = np.zeros((L, world), np.int64)
+        _native.check(f(ctypes.byref(s), capacity, world, ctypes.byref(nl), off.ctypes.data, rows.ctypes.data,
+                        early.ctypes.data))
+        levels = [(self.n_inputs + int(off[k]), int(off[k + 1] - off[k])) for k in range(L)]
+        return levels, rows, early
+
 
 # ------------------------------------------------------------------------------------- binary format
 def _inst(hi62: int, mid62: int, t4: int) -> bytes:

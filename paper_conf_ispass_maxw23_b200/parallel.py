@@ -43,20 +43,37 @@ def barrier(group, device=None):
         dist.barrier(group=group)
 
 
-def level_loop(levels, wires, run_level, group=None, fused=False):
+def level_loop(levels, wires, run_level, group=None, fused=False, early=None):
     """levels: [(row0, n_gates)] for levels 1..L; run_level(level, g0, g1) evaluates a gate range of a level
     into `wires` (a [rows, stride] tensor).  With a process group of R > 1 ranks every level's output rows must
     reach all ranks before the next level: fused=True means run_level's kernels already stored them into every
-    rank's array (fused all-gather), so only a barrier is taken; otherwise they are all-gathered in place."""
+    rank's array (fused all-gather), so only a barrier is taken; otherwise they are all-gathered in place.
+
+    early: per level, how many gates at the start of this rank's chunk read only rows that are
+    already local once this rank has run its own part of the previous level (a netlist planned for R ranks,
+    tb_set_plan_world).  Those gates run before the previous level's exchange, so the exchange and its barrier
+    overlap this rank's next work:  run the rest of level L, run the early part of level L + 1, exchange L."""
     import torch.distributed as dist
     R = dist.get_world_size(group) if group is not None else 1
     r = dist.get_rank(group) if group is not None else 0
+    nL = len(levels)
+    if not fused:
+        # the padded all-gather of level L writes R * chunk rows, i.e. also the first rows of level L + 1: gates of
+        # level L + 1 evaluated before it would be overwritten.  Early start needs the fused exchange.
+        early = None
     for L, (row0, ng) in enumerate(levels, start=1):
         g0, g1, chunk = shard(ng, R, r)
         if R > 1 and not fused and row0 + R * chunk > wires.shape[0]:
             raise ValueError("wire array needs slack rows for the padded all-gather (see slack_rows)")
-        if g1 > g0:
-            run_level(L, g0, g1)
+        # level 1 reads only inputs; later levels: their early part already ran before the previous exchange
+        start = g0 if (early is None or L == 1) else min(g0 + int(early[L - 1]), g1)
+        if g1 > start:
+            run_level(L, start, g1)
+        if early is not None and L < nL:                    # the next level's locally ready gates, before exchange L
+            ra, rb, _ = shard(levels[L][1], R, r)
+            e = min(int(early[L]), rb - ra)
+            if e > 0:
+                run_level(L + 1, ra, ra + e)
         if R > 1 and chunk:
             if fused:
                 barrier(group, wires.device)

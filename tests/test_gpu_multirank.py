@@ -32,7 +32,7 @@ def _netlist():
     return dict(n_inputs=n_in, type=t, in0=a, in1=b, in2=c)
 
 
-def _worker(rank, world, port, keyfile, ctsfile, q, exchange):
+def _worker(rank, world, port, keyfile, ctsfile, q, exchange, early_start=False):
     import torch
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -45,7 +45,7 @@ def _worker(rank, world, port, keyfile, ctsfile, q, exchange):
         ctx.load_keys(k["bk"], k["ksk"])
         n = _netlist()
         net = tb.Netlist(n["n_inputs"], n["type"], n["in0"], n["in1"], n["in2"])
-        dnet = ctx.upload(net)
+        dnet = ctx.upload(net, world=world if early_start else 1)   # early start: level order for R ranks
         wires = ctx.wire_array(dnet, slack_rows=tb.slack_rows(dnet, world))
         cts = np.load(ctsfile)
         wires[:n["n_inputs"], :631] = ctx.to_device(cts)[:, :631]
@@ -56,10 +56,14 @@ def _worker(rank, world, port, keyfile, ctsfile, q, exchange):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,exchange", [(2, "allgather"), (3, "allgather"), (2, "fused"), (3, "fused")])
-def test_sharded_netlist_matches_oracle(world, exchange):
+@pytest.mark.parametrize("world,exchange,early", [(2, "allgather", False), (3, "allgather", False),
+                                                  (2, "fused", False), (3, "fused", False), (2, "fused", True),
+                                                  (3, "fused", True)])
+def test_sharded_netlist_matches_oracle(world, exchange, early):
     """exchange="fused": the key-switch kernels store each output row into every rank's wire array through CUDA
-    IPC peer mappings (the fused all-gather; same-device IPC between processes here, NVLink peers on a box)"""
+    IPC peer mappings (the fused all-gather; same-device IPC between processes here, NVLink peers on a box).
+    early=True: the netlist is planned for R ranks and each rank runs the next level's locally ready gates
+    before the current level's barrier."""
     import torch
     import torch.multiprocessing as mp
     if not torch.cuda.is_available():
@@ -76,7 +80,8 @@ def test_sharded_netlist_matches_oracle(world, exchange):
         ctx = mp.get_context("spawn")
         q = ctx.Queue()
         port = _port()
-        procs = [ctx.Process(target=_worker, args=(r, world, port, kf, cf, q, exchange)) for r in range(world)]
+        procs = [ctx.Process(target=_worker, args=(r, world, port, kf, cf, q, exchange, early))
+                 for r in range(world)]
         for p in procs:
             p.start()
         res = [q.get(timeout=600) for _ in range(world)]

@@ -127,6 +127,29 @@ def test_run_netlist_host_matches_device(tb, ctx, keys):
     assert (ctx.run_netlist_host(dnet, wide, np.array([0, n["n_inputs"]])) == ref[[0, n["n_inputs"]]]).all()
 
 
+def test_run_netlist_host_overlap_equals_serial(tb, ctx, keys):
+    """tb_run_netlist_host with its copies overlapped with the level loop (inputs in first-use order on one
+    stream, each level's outputs copied back on another while the next level runs) gives the same
+    bytes as the serial path and as the device path: outputs from every level, inputs passed through, reversed
+    order, pinned and pageable host buffers"""
+    import torch
+    n = synth.array_multiplier(8, full=True)
+    cts = O.encrypt_bits(keys, synth.random_bits(n["n_inputs"], 15), 16)
+    ref, dnet = run(tb, ctx, n, cts)
+    ow = np.arange(dnet.n_rows - 1, -1, -3, dtype=np.int64)          # every third wire, reversed, incl. inputs
+    hin = torch.from_numpy(np.ascontiguousarray(cts).view(np.int32)).pin_memory()
+    outs = []
+    for overlap in (True, False):
+        ctx.set_host_overlap(overlap)
+        hout = torch.zeros((ow.size, 631), dtype=torch.int32).pin_memory()
+        ctx.run_netlist_host_into(dnet, hin, ow, hout)
+        outs.append(hout.numpy().view(np.uint32).copy())
+        outs.append(ctx.run_netlist_host(dnet, cts, ow))                 # pageable numpy buffers
+    ctx.set_host_overlap(True)
+    for o in outs:
+        assert (o == ref[ow]).all()
+
+
 def test_same_wire_twice_and_duplicate_consumers(tb, ctx, keys):
     """XOR(a, a) = 0 and AND(a, a) = a; one wire feeding many gates of a level"""
     n = dict(n_inputs=2, type=np.array([6, 8, 7, 7, 14], np.int32), in0=np.array([0, 0, 0, 1, 2]),
