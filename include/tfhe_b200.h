@@ -67,8 +67,11 @@ int tb_ctx_create(const tb_params* params, int cuda_device, tb_ctx** out);
 int tb_ctx_destroy(tb_ctx* ctx);
 
 /* Bootstrapping key, HOST pointer, torus layout [i < n][row r = bloc*l + j < 2l][poly < 2][N] u32
- * (n_words must equal n*2l*2*N = 7,741,440).  The library splits each coefficient into 3 signed parts,
- * transforms them to the NTT domain on the device (92.9 MB resident) and keeps no host copy.  Synchronous. */
+ * (n_words must equal n*2l*2*N = 7,741,440).  The torus key stays on the device (31 MB) and only the transform
+ * domains that the selected kernels read are built from it: the NTT domain (br6 / br9: each coefficient split
+ * into 3 signed parts, 92.9 MB), the FFT domain (brf / brl, 123.9 MB), the four-step NTT domain (brt, 92.9 MB).
+ * Selecting another kernel later (tb_set_br_variant / tb_set_narrow_kernel / tb_set_narrow_lanes) builds the
+ * domains it needs then (synchronously).  No host copy is kept.  Synchronous. */
 int tb_load_bk(tb_ctx* ctx, const uint32_t* host_bk, size_t n_words);
 /* Key-switching key, HOST pointer, layout [i < N][j < t][d < 4][n+1] u32 (n_words = 10,338,304).  Digit-0
  * rows (encryptions of 0, never read, C9) are dropped and rows padded to 632 words (62.1 MB).  Synchronous. */
@@ -230,7 +233,7 @@ int tb_netlist_world(const tb_dev_netlist* dnet, int* world);
 int tb_netlist_early(const tb_dev_netlist* dnet, int64_t level, int rank, int64_t* n_early);
 /* Gates per key-switch CTA (8, 16 or 32; default 8): each tile streams the 62 MB KSK once from L2. */
 int tb_set_ks_tile(tb_ctx* ctx, int gates);
-/* Device bytes a context holds for keys (BK NTT + KSK). */
+/* Device bytes a context holds for keys: the torus BK, the BK domains built so far, the KSK. */
 int tb_key_bytes(const tb_ctx* ctx, size_t* bytes);
 
 /* Integer-pipe microbenchmark (roofline denominator): runs the kernels' own lazy

@@ -89,6 +89,8 @@ struct tb_ctx {
     double2* bkf = nullptr;                 // FP64 variant: [n][6][4][512] complex, scaled by 1/512
     uint32_t* ksk = nullptr;                // [N][t][3][632]
     bool have_bk = false, have_ksk = false;
+    uint32_t* bk_raw = nullptr;             // the torus BK as loaded (31 MB): source of every domain built later
+    unsigned domains = 0;                   // BK domains built from bk_raw (kDomNtt | kDomFft | kDomBk4)
     // scratch (grown on demand; growing synchronises the device)
     uint32_t* lanebuf = nullptr;
     int64_t lanebuf_rows = 0;
@@ -292,6 +294,7 @@ extern "C" int tb_ctx_destroy(tb_ctx* c) {
     cudaFree(c->fftC);
     cudaFree(c->fftL);
     cudaFree(c->bkhat);
+    cudaFree(c->bk_raw);
     cudaFree(c->bk4);
     cudaFree(c->tcB);
     cudaFree(c->tcTw);
@@ -343,18 +346,46 @@ extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
     return TB_OK;
 }
 
+// ---- BK domains: only those the selected kernels read are built (from the loaded torus BK) ----------------
+enum : unsigned { kDomNtt = 1, kDomFft = 2, kDomBk4 = 4 };
+static unsigned needed_domains(const tb_ctx* c) {
+    unsigned m = c->variant == 10 ? kDomFft : (c->variant == 12 ? kDomBk4 : kDomNtt);
+    if (c->narrow_lanes > 0) {                         // latency mode: brl (FFT domain) and / or br9 (NTT domain)
+        if (c->narrow_kernel == 9) m |= kDomNtt;
+        else if (c->narrow_kernel == 11) m |= kDomFft;
+        else m |= kDomNtt | kDomFft;                   // auto: brl while the lanes fit one wave, else br9
+    }
+    return m;
+}
+static int build_domains(tb_ctx* c) {
+    if (!c->have_bk) return TB_OK;
+    const unsigned miss = needed_domains(c) & ~c->domains;
+    if (!miss) return TB_OK;
+    TB_CUDA(cudaSetDevice(c->device));
+    if ((miss & kDomNtt) && !c->bkhat) TB_CUDA(cudaMalloc(&c->bkhat, (size_t)kn * kRows * kOuts * kN * 4));
+    if ((miss & kDomFft) && !c->bkf) TB_CUDA(cudaMalloc(&c->bkf, bkf_bytes()));
+    if ((miss & kDomBk4) && !c->bk4) TB_CUDA(cudaMalloc(&c->bk4, bk4_bytes()));
+    if (miss & kDomNtt) launch_bk_to_ntt(c->bk_raw, c->bkhat, c->twF, c->ninv, c->ninvp, c->own);
+    if (miss & kDomFft) launch_bk_to_fft(c->bk_raw, c->bkf, c->fftB, c->fftC, c->own);
+    if (miss & kDomBk4) launch_bk_to_bk4(c->bk_raw, c->bk4, c->tcPts, c->ninv, c->ninvp, kn, c->own);
+    TB_CUDA(cudaGetLastError());
+    TB_CUDA(cudaStreamSynchronize(c->own));
+    c->domains |= miss;
+    return TB_OK;
+}
+
 extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
     if (!c || !(variant == 6 || variant == 10 || variant == 12))
         return fail(TB_EINVAL, "blind-rotation variant must be 6, 10 or 12");
     c->variant = variant;
-    return TB_OK;
+    return build_domains(c);
 }
 
 extern "C" int tb_set_narrow_kernel(tb_ctx* c, int kernel) {
     if (!c || (kernel != 0 && kernel != 9 && kernel != 11))
         return fail(TB_EINVAL, "latency-mode kernel must be 0 (auto), 9 or 11");
     c->narrow_kernel = kernel;
-    return TB_OK;
+    return build_domains(c);
 }
 
 extern "C" int tb_set_level_capacity(tb_ctx* c, int64_t lanes) {
@@ -366,7 +397,7 @@ extern "C" int tb_set_level_capacity(tb_ctx* c, int64_t lanes) {
 extern "C" int tb_set_narrow_lanes(tb_ctx* c, int64_t lanes) {
     if (!c || lanes < 0) return fail(TB_EINVAL, "narrow-level threshold must be >= 0");
     c->narrow_lanes = lanes;
-    return TB_OK;
+    return build_domains(c);
 }
 
 extern "C" int tb_set_plan_world(tb_ctx* c, int world) {
@@ -397,7 +428,9 @@ extern "C" int tb_set_ks_tile(tb_ctx* c, int gates) {
 
 extern "C" int tb_key_bytes(const tb_ctx* c, size_t* bytes) {
     if (!c || !bytes) return fail(TB_EINVAL, "null argument");
-    *bytes = (c->have_bk ? (size_t)kn * kRows * kOuts * kN * 4 : 0) +
+    *bytes = (c->have_bk ? (size_t)kn * kRows * 2 * kN * 4 : 0) +                       // torus BK (source)
+             ((c->domains & kDomNtt) ? (size_t)kn * kRows * kOuts * kN * 4 : 0) +
+             ((c->domains & kDomFft) ? bkf_bytes() : 0) + ((c->domains & kDomBk4) ? bk4_bytes() : 0) +
              (c->have_ksk ? (size_t)kN * kKsT * (kKsBase - 1) * kKsRow * 4 : 0);
     return TB_OK;
 }
@@ -407,23 +440,12 @@ extern "C" int tb_load_bk(tb_ctx* c, const uint32_t* host_bk, size_t n_words) {
     const size_t want = (size_t)kn * kRows * 2 * kN;
     if (n_words != want) return fail(TB_EINVAL, "bootstrapping key must have n*2l*2*N words");
     TB_CUDA(cudaSetDevice(c->device));
-    if (!c->bkhat) TB_CUDA(cudaMalloc(&c->bkhat, (size_t)kn * kRows * kOuts * kN * 4));
-    if (!c->bkf) TB_CUDA(cudaMalloc(&c->bkf, bkf_bytes()));
-    if (!c->bk4) TB_CUDA(cudaMalloc(&c->bk4, bk4_bytes()));
-    uint32_t* tmp = nullptr;
-    TB_CUDA(cudaMalloc(&tmp, want * 4));
-    cudaError_t e = cudaMemcpyAsync(tmp, host_bk, want * 4, cudaMemcpyHostToDevice, c->own);
-    if (e == cudaSuccess) {
-        launch_bk_to_ntt(tmp, c->bkhat, c->twF, c->ninv, c->ninvp, c->own);
-        launch_bk_to_fft(tmp, c->bkf, c->fftB, c->fftC, c->own);
-        launch_bk_to_bk4(tmp, c->bk4, c->tcPts, c->ninv, c->ninvp, kn, c->own);
-        e = cudaGetLastError();
-    }
-    if (e == cudaSuccess) e = cudaStreamSynchronize(c->own);
-    cudaFree(tmp);
-    if (e != cudaSuccess) return cuda_fail(e, "tb_load_bk");
+    if (!c->bk_raw) TB_CUDA(cudaMalloc(&c->bk_raw, want * 4));
+    TB_CUDA(cudaMemcpyAsync(c->bk_raw, host_bk, want * 4, cudaMemcpyHostToDevice, c->own));
+    TB_CUDA(cudaStreamSynchronize(c->own));
     c->have_bk = true;
-    return TB_OK;
+    c->domains = 0;                                  // a new key: every domain is rebuilt from it
+    return build_domains(c);
 }
 
 extern "C" int tb_load_ksk(tb_ctx* c, const uint32_t* host_ksk, size_t n_words) {

@@ -63,3 +63,26 @@ def test_tc_muladd_equals_schoolbook(ctx):
                 for r in range(6):
                     want = O.negacyclic_muladd(d32[g, r], b32[r, q], want)
                 assert (got[g, q] == want).all(), (g, q)
+
+
+def test_bk_domains_built_on_demand():
+    """only the BK domains the selected kernels read are resident: the tensor-core domain
+    appears when variant 12 is selected after the load, and its kernel is then bit-exact"""
+    import torch
+    import oracle as O
+    import paper_conf_ispass_maxw23_b200 as tb
+    keys = O.keygen(O.DEFAULT, seed=31)
+    c = tb.Context(0)
+    try:
+        c.load_keys(keys.bk, keys.ksk)
+        before = c.key_bytes()
+        c.set_br_variant(12)
+        after = c.key_bytes()
+        assert after - before == 630 * 1024 * 36 * 4                    # the four-step domain, 92.9 MB
+        c.set_narrow_lanes(0)
+        cts = O.encrypt_bits(keys, [1, 0, 1], 32)
+        got = c.bootstrap_wo_ks(c.to_device(cts))[:, :1025].cpu().numpy().view(np.uint32)
+        for k in range(3):
+            assert (got[k] == O.bootstrap_wo_ks(keys, cts[k])).all()
+    finally:
+        c.close()
