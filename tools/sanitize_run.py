@@ -1,7 +1,9 @@
 #!/usr/bin/env python
-"""Small run of every kernel (all blind-rotation variants, every latency-mode kernel, tiled and split key
-switch at 3 / 7 / 37 gates, a mixed netlist, and the fused-exchange peer stores into a second array) for
-compute-sanitizer:  compute-sanitizer --tool {memcheck,racecheck,synccheck} python tools/sanitize_run.py"""
+"""Small run of every kernel (all blind-rotation variants incl. the tensor-core brt, every latency-mode kernel,
+tiled and split key switch at 3 / 7 / 37 gates, a mixed netlist through the device and the overlapped host path,
+and the fused-exchange peer stores into a second array) for compute-sanitizer:
+    compute-sanitizer --tool {memcheck,racecheck,synccheck} python tools/sanitize_run.py
+TB_SAN_BRT=1: only the tensor-core kernel (racecheck on its shared-memory hand-offs)."""
 import ctypes
 import os
 import sys
@@ -22,6 +24,17 @@ ct.random_(-2 ** 31, 2 ** 31 - 1, generator=g)
 outs = []
 QUICK = os.environ.get("TB_SAN_QUICK") == "1"                # racecheck: key switch, netlist and peer stores only
 LAT = os.environ.get("TB_SAN_LATENCY") == "1"                # racecheck: the latency kernels on one lane only
+BRT = os.environ.get("TB_SAN_BRT") == "1"                    # racecheck: the tensor-core kernel only
+if BRT:
+    ctx.set_narrow_lanes(0)
+    ctx.set_br_variant(6)
+    a = ctx.bootstrap_wo_ks(ct)
+    ctx.set_br_variant(12)
+    b = ctx.bootstrap_wo_ks(ct)
+    torch.cuda.synchronize()
+    ok = torch.equal(a[:, :1025], b[:, :1025])
+    print("brt agrees with br6:", ok)
+    sys.exit(0 if ok else 1)
 if LAT:
     one = ct[:1]
     res = []
@@ -32,7 +45,7 @@ if LAT:
     ok = torch.equal(res[0][:, :1025], res[1][:, :1025])
     print("latency kernels agree:", ok)
     sys.exit(0 if ok else 1)
-for variant in ((6,) if QUICK else (6, 10)):
+for variant in ((6,) if QUICK else (6, 10, 12)):
     ctx.set_br_variant(variant)
     ctx.set_narrow_lanes(0)
     outs.append(ctx.bootstrap_wo_ks(ct))
@@ -54,6 +67,8 @@ d = ctx.upload(net)
 w = ctx.wire_array(d)
 w[:n["n_inputs"]].random_(-2 ** 31, 2 ** 31 - 1, generator=g)
 ctx.run_netlist(d, w)
+hin = w[:n["n_inputs"], :631].cpu().contiguous()
+hout = ctx.run_netlist_host(d, hin.numpy().view("uint32"), [d.n_rows - 1, 0])   # overlapped host path
 mirror = ctx.wire_array(d)                                  # fused exchange: peer stores into a second array
 arr = (ctypes.c_void_p * 1)(mirror.data_ptr())
 tb._native.check(tb._native.lib().tb_set_peer_wires(ctx._h, ctypes.c_void_p(w.data_ptr()), arr, 1))
