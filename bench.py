@@ -225,6 +225,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-sweep", action="store_true", help="skip the 1 K - 256 K gates-per-level sweep")
     ap.add_argument("--one-gpu-ranks", action="store_true",
                     help="functional check of the N > 1 path on a one-GPU box: every rank on cuda:0, gloo process "
                          "group (the numbers are not a scaling measurement)")
@@ -416,6 +417,30 @@ def main():
     ctx.profile(False)
     lat_roof = latency_roofline(lat, lks_ms / max(lks_n, 1), clk_mhz, 11)
 
+    # throughput sweep of BASELINE configs[2] (1 K - 256 K independent gates per level, this GPU alone): device time
+    # of one level per point, median of 2 after a warm-up (the headline `value` is the 65,536-gate point above)
+    sweep = None
+    if group is None and not args.no_sweep:
+        sweep = {}
+        for Gs in (1024, 4096, 16384, 262144):
+            ns = synth.independent_level(Gs, seed=16)
+            snet = ctx.upload(tb.Netlist(ns["n_inputs"], ns["type"], ns["in0"], ns["in1"], ns["in2"]))
+            sw = ctx.wire_array(snet)
+            sw[:ns["n_inputs"]].random_(-2 ** 31, 2 ** 31 - 1, generator=gen)
+            ctx.run_netlist(snet, sw)
+            times = []
+            for _ in range(2):
+                s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                s0.record()
+                ctx.run_netlist(snet, sw)
+                s1.record()
+                torch.cuda.synchronize()
+                times.append(s0.elapsed_time(s1))
+            sweep[str(Gs)] = {"level_ms": statistics.median(times), "gates_per_s": Gs / (statistics.median(times) / 1e3)}
+            del sw
+            snet.free()
+        sweep[str(G)] = {"level_ms": ms / args.steps, "gates_per_s": G * args.steps / (ms / 1e3)}
+
     # e2e through the public API with host buffers: N = 1 the C ABI's tb_run_netlist_host; N > 1 the sharded
     # level loop (each rank copies in the input rows its gates read, runs its shard with the level exchange,
     # copies back the outputs it produced)
@@ -506,7 +531,7 @@ def main():
             "roofline": roofline, "latency_roofline": lat_roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
             "gpu_launches": br_n + ks_n,
             "latency_ms": {"level_of_%d_gates" % total: ms / args.steps, "level_of_1_gate": lat},
-            "exchange": exch,
+            "exchange": exch, "sweep": sweep,
         }), flush=True)
     if group is not None:
         dist.barrier()
