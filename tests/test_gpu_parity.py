@@ -179,6 +179,23 @@ def test_keyswitch_bit_exact(tb, ctx, keys, narrow, count):
         assert (got[r] == O.keyswitch(keys, ext[r])).all(), r
 
 
+def test_keyswitch_split_scratch_nondefault_threshold(tb, keys):
+    """with a non-default narrow-level threshold (10) on a fresh context, a 9-gate split key switch
+    writes 9 x 32 partial rows (more than 10 x 16): the scratch is sized from the launch, results bit-exact"""
+    c = tb.Context(0)
+    try:
+        c.load_keys(keys.bk, keys.ksk)
+        c.set_narrow_lanes(10)
+        rng = np.random.default_rng(61)
+        for count in (9, 4, 10):
+            ext = rng.integers(0, M32, (count, 1025), dtype=np.uint64).astype(np.uint32)
+            got = c.to_host(c.keyswitch(c.to_device(ext, stride=1028)))
+            for r in range(count):
+                assert (got[r] == O.keyswitch(keys, ext[r])).all(), (count, r)
+    finally:
+        c.close()
+
+
 # ------------------------------------------------------------------------------------- gates
 def test_nand_truth_table_config1(tb, ctx, keys):
     """BASELINE configs[0]: NAND truth table, 4 bootstraps, bit-exact and decrypting to 1,1,1,0."""
