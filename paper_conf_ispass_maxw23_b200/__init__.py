@@ -410,16 +410,22 @@ class Context:
                 mine.append(np.arange(row0 - ni + g0, row0 - ni + g1))
         pos = np.concatenate(mine) if mine else np.zeros(0, np.int64)
         g = order[pos]
-        ins = np.concatenate([net.in0[g], net.in1[g], net.in2[g]])
-        in_rows = np.unique(ins[(ins >= 0) & (ins < ni)])
+        ins = np.concatenate([net.in0[g], np.where(net.type[g] == NOT, -1, net.in1[g]),
+                              np.where(net.type[g] == MUX, net.in2[g], -1)])
+        ins = ins[(ins >= 0) & (ins < ni)]
         outs = []
         if output_wires is not None:
             ow = np.asarray(output_wires, np.int64)
             rows = dnet.row_of_wire[ow]
             produced = np.zeros(dnet.n_rows, bool)
             produced[ni + pos] = True
+            if rank == 0:                    # outputs that are primary inputs (passed through): rank 0 returns them
+                produced[:ni] = True
             k = np.nonzero(produced[rows])[0]
             outs = list(zip(k.tolist(), rows[k].tolist()))
+            if rank == 0:
+                ins = np.concatenate([ins, rows[rows < ni]])
+        in_rows = np.unique(ins)
         cache[key] = (in_rows, outs)
         return cache[key]
 

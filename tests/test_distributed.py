@@ -212,3 +212,38 @@ def test_shard_and_slack():
             spans = [parallel.shard(ng, R, r) for r in range(R)]
             assert sum(g1 - g0 for g0, g1, _ in spans) == ng
             assert all(spans[r][1] == spans[r + 1][0] for r in range(R - 1))
+
+
+def test_shard_io_covers_inputs_and_outputs_once():
+    """Context.shard_io (the per-rank I/O plan of the sharded end-to-end path, run_netlist_host_sharded): every
+    rank's input rows contain every primary input its gate ranges read, and over the ranks every requested output
+    is returned exactly once -- by the rank that produced it, or by rank 0 for an input passed through (host
+    logic, no GPU)"""
+    from types import SimpleNamespace
+
+    import paper_conf_ispass_maxw23_b200 as tb
+    from paper_conf_ispass_maxw23_b200 import parallel
+    for seed in range(3):
+        n_in, t, a, b, c = _netlist(seed)
+        net = tb.Netlist(n_in, t, a, b, c)
+        lv, rows = net.plan()
+        dnet = SimpleNamespace(net=net, row_of_wire=rows, n_rows=net.n_wires,
+                               levels=[(row0, ng, 0, 0) for row0, ng in lv])
+        outs = np.random.default_rng(seed).choice(net.n_wires, 25, replace=False)
+        order = np.argsort(rows[n_in:])
+        for world in (1, 2, 3):
+            seen = []
+            for r in range(world):
+                in_rows, o = tb.Context.shard_io(None, dnet, world, r, outs)
+                seen += [k for k, _ in o]
+                assert all(rows[outs[k]] == row for k, row in o)
+                for row0, ng in lv:
+                    g0, g1, _ = parallel.shard(ng, world, r)
+                    for k in range(row0 - n_in + g0, row0 - n_in + g1):
+                        g = order[k]
+                        for w in (a[g], b[g], c[g]):
+                            if 0 <= w < n_in and (w != b[g] or t[g] != 3) and (w != c[g] or t[g] == 16):
+                                assert w in in_rows
+            assert sorted(seen) == list(range(outs.size))      # pass-through inputs come from rank 0
+            in0, _ = tb.Context.shard_io(None, dnet, world, 0, outs)
+            assert all(rows[w] in in0 for w in outs if rows[w] < n_in)
