@@ -80,11 +80,19 @@ __device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
 // try_wait with a suspend-time hint: a waiting thread sleeps in the barrier instead of re-issuing the test
 // (the spinning MMA thread otherwise takes issue slots from the compute warps of its sub-partition)
 __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+#ifdef TB_NO_SUSPEND_HINT
+    asm volatile(
+        "{\n .reg .pred p;\n TCW_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        " @!p bra TCW_%=;\n}\n" ::"r"(smem_u32(b)),
+        "r"(parity)
+        : "memory");
+#else
     asm volatile(
         "{\n .reg .pred p;\n TCW_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
         " @!p bra TCW_%=;\n}\n" ::"r"(smem_u32(b)),
         "r"(parity), "r"(0x100000u)
         : "memory");
+#endif
 }
 
 // byte offset of (row, kbyte) in a K-major no-swizzle tile with the given core-matrix strides
