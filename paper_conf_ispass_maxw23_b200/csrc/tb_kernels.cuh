@@ -95,6 +95,7 @@ int brl_wave_lanes();
 namespace tb {
 // tensor-core blind rotation (tb_brt.cu)
 int launch_brt(const BrArgs& A, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw, cudaStream_t st);
+int launch_brtl(const BrArgs& A, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw, cudaStream_t st);
 int launch_brt_muladd(const int32_t* digits, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw,
                       uint32_t* res, cudaStream_t st);
 void launch_bk_to_bk4(const uint32_t* bk, uint32_t* bk4, const uint2* pts, uint32_t ninv, uint32_t ninvp, int n_i,

@@ -353,6 +353,7 @@ static unsigned needed_domains(const tb_ctx* c) {
     if (c->narrow_lanes > 0) {                         // latency mode: brl (FFT domain) and / or br9 (NTT domain)
         if (c->narrow_kernel == 9) m |= kDomNtt;
         else if (c->narrow_kernel == 11) m |= kDomFft;
+        else if (c->narrow_kernel == 13) m |= kDomBk4;
         else m |= kDomNtt | kDomFft;                   // auto: brl while the lanes fit one wave, else br9
     }
     return m;
@@ -382,8 +383,8 @@ extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
 }
 
 extern "C" int tb_set_narrow_kernel(tb_ctx* c, int kernel) {
-    if (!c || (kernel != 0 && kernel != 9 && kernel != 11))
-        return fail(TB_EINVAL, "latency-mode kernel must be 0 (auto), 9 or 11");
+    if (!c || (kernel != 0 && kernel != 9 && kernel != 11 && kernel != 13))
+        return fail(TB_EINVAL, "latency-mode kernel must be 0 (auto), 9, 11 or 13");
     c->narrow_kernel = kernel;
     return build_domains(c);
 }
@@ -512,8 +513,9 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
         nk = nlanes <= c->brl_wave ? 11 : 9;
     }
     if (c->narrow_lanes > 0 && nlanes <= c->narrow_lanes)
-        rc = nk == 9 ? launch_br9(A, st)                       // narrow level: one lane per 2-SM cluster
-                     : launch_brl(A, c->bkf, c->fftL, st);     // or per 4-SM cluster (FP64)
+        rc = nk == 9    ? launch_br9(A, st)                    // narrow level: one lane per 2-SM cluster
+             : nk == 13 ? launch_brtl(A, c->bk4, c->tcB, c->tcTw, st)   // or per SM on the tensor cores
+                        : launch_brl(A, c->bkf, c->fftL, st);  // or per 4-SM cluster (FP64)
     else if (c->variant == 12)
         rc = launch_brt(A, c->bk4, c->tcB, c->tcTw, st);
     else if (c->variant == 10)

@@ -96,10 +96,11 @@ def oracle_bootstrap_many(keys, cts):
         return np.stack(list(ex.map(lambda c: O.bootstrap_wo_ks(keys, c), cts)))
 
 
-@pytest.mark.parametrize("kernel", [0, 9, 11])
+@pytest.mark.parametrize("kernel", [0, 9, 11, 13])
 def test_narrow_level_latency_mode_bit_exact(tb, ctx, keys, kernel):
     """small launches run the latency kernel (br9: 2-SM cluster per lane, brl: 4-SM cluster per lane on the
-    FP64 path; 40 lanes = 160 CTAs is more than one wave of brl); 149 lanes fall back to the throughput kernel.
+    FP64 path, brtl: one SM per lane on the tensor cores; 40 lanes = 160 CTAs is more than one wave of brl);
+    149 lanes fall back to the throughput kernel.
     Every lane of the 1-, 3- and 40-lane launches is compared with the oracle, the first and last of 149."""
     rng = np.random.default_rng(39 + kernel)
     ctx.set_narrow_kernel(kernel)
