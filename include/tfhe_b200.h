@@ -201,11 +201,12 @@ int tb_set_br_variant(tb_ctx* ctx, int variant);
 /* Latency mode for narrow levels: a launch with <= `lanes` bootstraps runs a latency-mode kernel (below)
  * instead of the throughput kernel.  Default = the device's SM count; 0 disables. */
 int tb_set_narrow_lanes(tb_ctx* ctx, int64_t lanes);
-/* Latency-mode kernel: 0 = auto (default: brl while the level's bootstraps fit in one wave of brl clusters,
- * else br9), 11 = brl_kernel (one bootstrap per cluster of 4 SMs on the FP64 path: each SM owns one output
- * polynomial and one 16-bit BK half, transforms split over warp pairs; 1.9 ms per level on B200),
- * 9 = br9_kernel (one bootstrap per cluster of 2 SMs, each SM owning one accumulator polynomial, forward-NTT
- * rows exchanged through distributed shared memory; 2.8 ms, 74 per wave).  Both are bit-identical.  Anything else: TB_EINVAL. */
+/* Latency-mode kernel: 0 = auto (default: brl while the level's bootstraps fit in one wave of brl clusters, br9
+ * while they fit one wave of its SM pairs, else brtl), 11 = brl_kernel (one bootstrap per cluster of 4 SMs on the
+ * FP64 path: each SM owns one output polynomial and one 16-bit BK half; 1.9 ms per level on B200, 32 per wave),
+ * 9 = br9_kernel (one bootstrap per cluster of 2 SMs, forward-NTT rows exchanged through distributed shared memory;
+ * 3.5 ms, 74 per wave), 13 = brtl_kernel (one bootstrap per SM on the tensor cores, tb_brtl.cu; 4.7 ms, 148 per
+ * wave).  All are bit-identical.  Anything else: TB_EINVAL. */
 int tb_set_narrow_kernel(tb_ctx* ctx, int kernel);
 /* Level schedule used by tb_netlist_upload: Algorithm 1 gives every gate its earliest level;
  * with lanes > 0 gates that have slack are moved to later levels (never past their latest level, so the number

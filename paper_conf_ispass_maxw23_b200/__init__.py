@@ -156,7 +156,7 @@ class Context:
         _native.check(_native.lib().tb_set_level_capacity(self._h, lanes))
 
     def set_narrow_kernel(self, kernel: int):
-        """latency-mode kernel: 0 = auto (default), 11 = brl (4-SM cluster), 9 = br9 (2-SM cluster)"""
+        """latency-mode kernel: 0 = auto (default), 11 = brl (4-SM cluster), 9 = br9 (2-SM cluster), 13 = brtl (1 SM, tensor cores)"""
         _native.check(_native.lib().tb_set_narrow_kernel(self._h, kernel))
 
     def set_ks_tile(self, gates: int):

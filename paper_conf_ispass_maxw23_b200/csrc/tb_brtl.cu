@@ -4,10 +4,12 @@
 // Same arithmetic as brt_kernel (tb_brt.cu): the four-step NTTs of the CMux as
 // tcgen05.mma.kind::i8 byte-limb GEMMs, the MAC against the four-step BK records, centred lift -- bit-identical to
 // every other variant.  What changes is the shape: one lane (6 + 6 polynomials = 2 M-tiles per stage) on a whole SM,
-// 16 warps, every stage synchronous (thread 0 issues, everyone waits on the commit), so that a CMux step costs the
-// latency of 4 small GEMMs + 4 short epilogues (16 values per thread) + a MAC over 2 coefficients per thread.  The
-// 36-word BK records of the step's MAC are requested at the top of the step, so their L2 latency hides behind the
-// forward half.  A level of <= 148 bootstraps runs in one wave (one CTA per SM).
+// 16 warps, every stage synchronous (thread 0 issues, everyone waits on the commit): a CMux step costs 4 small GEMMs
+// + 4 short epilogues (16 values per thread) + a MAC over 2 coefficients per thread.  A level of <= 148 bootstraps
+// runs in one wave (one CTA per SM): 4.6-4.7 ms for 1-148 bootstraps on B200, which beats br9 from ~75 bootstraps
+// on; a single gate stays faster on brl (1.9 ms), whose 4 SMs share the step's BK stream (one SM must ingest the
+// whole 147 KB of BK records per step here; requesting them at the top of the step was measured slower, 5.3 ms:
+// the 18 16-byte loads per thread throttle the load queue and the registers they hold spill).
 #include "tb_kernels.cuh"
 #include "tb_ntt.cuh"
 #include "tb_tc.cuh"
@@ -16,7 +18,10 @@ namespace tb {
 
 constexpr int kTlWarps = 16;
 constexpr int kTlThreads = 32 * kTlWarps;
-constexpr int kTlTiles = 2;                   // polys 0-3 and 4-5 (rows 64-127 of tile 1 are padding)
+constexpr int kTlTiles = 2;
+#ifndef TB_BRTL_BK
+#define TB_BRTL_BK 0                          // BK records: 0 = all at the top of the step, 1 = split, 2 = in the MAC
+#endif                   // polys 0-3 and 4-5 (rows 64-127 of tile 1 are padding)
 
 struct BrtlSmem {
     unsigned char B[kTcBTotal];               // constant B operands (the same as brt_kernel's)
@@ -113,11 +118,6 @@ __global__ void __launch_bounds__(kTlThreads, 1) brtl_kernel(BrArgs A, const uin
     for (int i = 0; i < kn; i++) {
         // ---- BK records of this step's MAC (positions tid, tid + 512), in flight during the forward half
         const uint4* rec = reinterpret_cast<const uint4*>(bk4 + ((size_t)i * kN + tid) * kBk4Rec);
-        uint4 Bk[2][kBk4Rec / 4];
-#pragma unroll
-        for (int h = 0; h < 2; h++)
-#pragma unroll
-            for (int q = 0; q < kBk4Rec / 4; q++) Bk[h][q] = __ldg(rec + h * 512 * (kBk4Rec / 4) + q);
         // ---- a4.1 digits of (X^abar - 1) ACC[bloc]: coefficients c = 32 (4 du4 + u) + lane, u < 4
         {
             const uint32_t ab = S.bar[i];
@@ -202,7 +202,8 @@ __global__ void __launch_bounds__(kTlThreads, 1) brtl_kernel(BrArgs A, const uin
                 uint32_t B[kBk4Rec];
 #pragma unroll
                 for (int q = 0; q < kBk4Rec / 4; q++) {
-                    B[4 * q] = Bk[h][q].x; B[4 * q + 1] = Bk[h][q].y; B[4 * q + 2] = Bk[h][q].z; B[4 * q + 3] = Bk[h][q].w;
+                    const uint4 b4 = __ldg(rec + h * 512 * (kBk4Rec / 4) + q);
+                    B[4 * q] = b4.x; B[4 * q + 1] = b4.y; B[4 * q + 2] = b4.z; B[4 * q + 3] = b4.w;
                 }
 #pragma unroll
                 for (int o = 0; o < 6; o++) {

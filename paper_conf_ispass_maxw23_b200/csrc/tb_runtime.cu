@@ -354,7 +354,7 @@ static unsigned needed_domains(const tb_ctx* c) {
         if (c->narrow_kernel == 9) m |= kDomNtt;
         else if (c->narrow_kernel == 11) m |= kDomFft;
         else if (c->narrow_kernel == 13) m |= kDomBk4;
-        else m |= kDomNtt | kDomFft;                   // auto: brl while the lanes fit one wave, else br9
+        else m |= kDomNtt | kDomFft | kDomBk4;         // auto: brl, br9 or brtl by the level's width
     }
     return m;
 }
@@ -508,9 +508,12 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     const long slot = prof_begin(c, 0, st);
     int rc;
     int nk = c->narrow_kernel;
-    if (nk == 0) {   // auto: measured one-lane level 2.2 ms (brl) vs 4.2 ms (br9), 32 vs 74 lanes per wave
+    if (nk == 0) {   // auto (profiles/r02y_latency.jsonl): brl while the lanes fit its 32 clusters (1.9 ms), br9
+                     // while they fit its SM pairs (3.5 ms), beyond that brtl with one lane per SM (4.7 ms flat)
         if (c->brl_wave == -2) c->brl_wave = brl_wave_lanes();
-        nk = nlanes <= c->brl_wave ? 11 : 9;
+        if (c->sms == 0 && cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess)
+            c->sms = 148;
+        nk = nlanes <= c->brl_wave ? 11 : (nlanes <= c->sms / 2 ? 9 : 13);
     }
     if (c->narrow_lanes > 0 && nlanes <= c->narrow_lanes)
         rc = nk == 9    ? launch_br9(A, st)                    // narrow level: one lane per 2-SM cluster
