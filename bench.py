@@ -217,7 +217,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--gates-per-gpu", type=int, default=65536)
     ap.add_argument("--lanes-per-cta", type=int, default=0, help="0 = auto per launch size")
-    ap.add_argument("--br-variant", type=int, default=6, choices=[6, 10, 12])
+    ap.add_argument("--br-variant", type=int, default=6, choices=[6, 10, 12, 14, 15])
     ap.add_argument("--ks-tile", type=int, default=8, choices=[8, 16, 32])
     ap.add_argument("--exchange", default="fused", choices=["fused", "allgather"],
                     help="N > 1: per-level exchange of output rows (fused into the key switch over NVLink peer "
@@ -371,7 +371,7 @@ def main():
             traffic = None
     roofline = {"bound": "alu", "achieved": achieved / 1e9, "peak": peak / 1e9, "unit": unit,
                 "frac": achieved / peak, "traffic": traffic,
-                "kernel": "%s (blind rotation + extraction)" % {10: "brf_kernel", 12: "brt_kernel"}.get(
+                "kernel": "%s (blind rotation + extraction)" % {10: "brf_kernel", 12: "brt_kernel", 14: "br6t_kernel", 15: "brq_kernel"}.get(
                     args.br_variant, "br%d_kernel" % args.br_variant),
                 "kernel_ms_per_launch": br_launch_s * 1e3,
                 "kernel_share_of_step": br_ms / ms if ms else None,

@@ -196,7 +196,9 @@ int tb_set_lanes_per_cta(tb_ctx* ctx, int lanes);
 int tb_br6_lanes_per_cta(tb_ctx* ctx, int64_t nlanes);
 /* Blind-rotation kernel: 6 = br6_kernel (default: 6 warps/lane, 2 CTAs/SM, BK words from L2), 10 = brf_kernel
  * (FP64-pipe FFT), 12 = brt_kernel (four-step NTT on the tcgen05 tensor cores, DESIGN.md
- * "Tensor-core NTT").  All are bit-identical; see DESIGN.md "Kernels".  Anything else: TB_EINVAL. */
+ * "Tensor-core NTT"), 14 = br6t_kernel (br6 with its forward NTTs on the tensor cores), 15 = brq_kernel (both
+ * NTT directions on the tensor cores in br6's 2-CTA-per-SM shape).  All are bit-identical; see
+ * DESIGN.md "Kernels".  Anything else: TB_EINVAL. */
 int tb_set_br_variant(tb_ctx* ctx, int variant);
 /* Latency mode for narrow levels: a launch with <= `lanes` bootstraps runs a latency-mode kernel (below)
  * instead of the throughput kernel.  Default = the device's SM count; 0 disables. */

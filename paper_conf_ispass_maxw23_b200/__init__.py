@@ -144,7 +144,8 @@ class Context:
         return rc
 
     def set_br_variant(self, variant: int):
-        """6 = br6_kernel (default), 10 = brf_kernel (FP64 pipe), 12 = brt_kernel (tensor cores); bit-identical."""
+        """6 = br6_kernel (default), 10 = brf_kernel (FP64 pipe), 12 = brt_kernel (tensor cores), 14 = br6t_kernel
+        (br6 with its forward NTT on the tensor cores); bit-identical."""
         _native.check(_native.lib().tb_set_br_variant(self._h, variant))
 
     def set_narrow_lanes(self, lanes: int):

@@ -95,6 +95,10 @@ int brl_wave_lanes();
 namespace tb {
 // tensor-core blind rotation (tb_brt.cu)
 int launch_brt(const BrArgs& A, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw, cudaStream_t st);
+// br6 with the forward NTT on the tensor cores (tb_br6t.cu): 2 lanes per CTA, NTT-domain BK (bkhat)
+int launch_br6t(const BrArgs& A, const unsigned char* tcB, const uint2* tcTw, cudaStream_t st);
+// both NTT directions on the tensor cores in br6's shape (tb_brq.cu): 2 lanes per CTA, natural-order BK (bk4)
+int launch_brq(const BrArgs& A, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw, cudaStream_t st);
 int launch_brtl(const BrArgs& A, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw, cudaStream_t st);
 int launch_brt_muladd(const int32_t* digits, const uint32_t* bk4, const unsigned char* tcB, const uint2* tcTw,
                       uint32_t* res, cudaStream_t st);

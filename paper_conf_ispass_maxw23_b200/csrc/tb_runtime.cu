@@ -349,7 +349,7 @@ extern "C" int tb_set_lanes_per_cta(tb_ctx* c, int lanes) {
 // ---- BK domains: only those the selected kernels read are built (from the loaded torus BK) ----------------
 enum : unsigned { kDomNtt = 1, kDomFft = 2, kDomBk4 = 4 };
 static unsigned needed_domains(const tb_ctx* c) {
-    unsigned m = c->variant == 10 ? kDomFft : (c->variant == 12 ? kDomBk4 : kDomNtt);
+    unsigned m = c->variant == 10 ? kDomFft : ((c->variant == 12 || c->variant == 15) ? kDomBk4 : kDomNtt);
     if (c->narrow_lanes > 0) {                         // latency mode: brl (FFT domain) and / or br9 (NTT domain)
         if (c->narrow_kernel == 9) m |= kDomNtt;
         else if (c->narrow_kernel == 11) m |= kDomFft;
@@ -376,8 +376,8 @@ static int build_domains(tb_ctx* c) {
 }
 
 extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
-    if (!c || !(variant == 6 || variant == 10 || variant == 12))
-        return fail(TB_EINVAL, "blind-rotation variant must be 6, 10 or 12");
+    if (!c || !(variant == 6 || variant == 10 || variant == 12 || variant == 14 || variant == 15))
+        return fail(TB_EINVAL, "blind-rotation variant must be 6, 10, 12, 14 or 15");
     c->variant = variant;
     return build_domains(c);
 }
@@ -521,6 +521,10 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
                         : launch_brl(A, c->bkf, c->fftL, st);  // or per 4-SM cluster (FP64)
     else if (c->variant == 12)
         rc = launch_brt(A, c->bk4, c->tcB, c->tcTw, st);
+    else if (c->variant == 14)
+        rc = launch_br6t(A, c->tcB, c->tcTw, st);
+    else if (c->variant == 15)
+        rc = launch_brq(A, c->bk4, c->tcB, c->tcTw, st);
     else if (c->variant == 10)
         rc = launch_brf(A, c->lanes_per_cta ? std::min(c->lanes_per_cta, 3) : 2, c->bkf, c->fftB, c->fftC, st);
     else

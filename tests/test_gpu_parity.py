@@ -114,7 +114,7 @@ def test_narrow_level_latency_mode_bit_exact(tb, ctx, keys, kernel):
         ctx.set_narrow_kernel(0)
 
 
-@pytest.mark.parametrize("variant", [6, 10, 12])
+@pytest.mark.parametrize("variant", [6, 10, 12, 14, 15])
 def test_blind_rotation_variants_bit_exact(tb, ctx, keys, variant):
     """every blind-rotation kernel variant (br6 integer NTT / brf FP64 FFT / brt tensor-core NTT) on a ragged
     batch of 9"""
@@ -394,7 +394,7 @@ def test_mixed_netlist_with_not_and_mux(tb, ctx, keys):
     assert (O.decrypt_bits(keys, gpu) == plain).all()
 
 
-@pytest.mark.parametrize("variant", [6, 10, 12])
+@pytest.mark.parametrize("variant", [6, 10, 12, 14, 15])
 def test_throughput_level_bench_size_sampled(tb, ctx, keys, variant):
     """BASELINE configs[2] at the bench's per-GPU size (65,536 NAND/XOR gates, one level, the launch
     configuration bench.py times, default br6 and --br-variant 10): all outputs decrypt to the truth; a
