@@ -3,7 +3,8 @@
 tiled and split key switch at 3 / 7 / 37 gates, a mixed netlist through the device and the overlapped host path,
 and the fused-exchange peer stores into a second array) for compute-sanitizer:
     compute-sanitizer --tool {memcheck,racecheck,synccheck} python tools/sanitize_run.py
-TB_SAN_BRT=1: only the tensor-core kernel (racecheck on its shared-memory hand-offs)."""
+TB_SAN_BRT=1: only the tensor-core kernels brt / br6t / brq / brtl (racecheck on their shared-memory hand-offs).
+TB_SAN_NOBRT=1: everything but the tensor-core kernels (synccheck does not model tcgen05.commit arrivals)."""
 import ctypes
 import os
 import sys
@@ -29,11 +30,17 @@ if BRT:
     ctx.set_narrow_lanes(0)
     ctx.set_br_variant(6)
     a = ctx.bootstrap_wo_ks(ct)
-    ctx.set_br_variant(12)
-    b = ctx.bootstrap_wo_ks(ct)
+    bs = []
+    for v in (12, 14, 15):
+        ctx.set_br_variant(v)
+        bs.append(ctx.bootstrap_wo_ks(ct))
+    ctx.set_br_variant(6)
+    ctx.set_narrow_lanes(148)
+    ctx.set_narrow_kernel(13)
+    bs.append(ctx.bootstrap_wo_ks(ct))
     torch.cuda.synchronize()
-    ok = torch.equal(a[:, :1025], b[:, :1025])
-    print("brt agrees with br6:", ok)
+    ok = all(torch.equal(a[:, :1025], b[:, :1025]) for b in bs)
+    print("brt / br6t / brq / brtl agree with br6:", ok)
     sys.exit(0 if ok else 1)
 if LAT:
     one = ct[:1]
@@ -46,13 +53,13 @@ if LAT:
     print("latency kernels agree:", ok)
     sys.exit(0 if ok else 1)
 NOBRT = os.environ.get("TB_SAN_NOBRT") == "1"                # synccheck: the tool does not model tcgen05.commit
-for variant in ((6,) if QUICK else ((6, 10) if NOBRT else (6, 10, 12))):
+for variant in ((6,) if QUICK else ((6, 10) if NOBRT else (6, 10, 12, 14, 15))):
     ctx.set_br_variant(variant)
     ctx.set_narrow_lanes(0)
     outs.append(ctx.bootstrap_wo_ks(ct))
 ctx.set_br_variant(6)
 ctx.set_narrow_lanes(148)
-for k in (() if QUICK else (11, 9)):                         # latency mode: brl, br9
+for k in (() if QUICK else ((11, 9) if NOBRT else (11, 9, 13))):   # latency mode: brl, br9, brtl
     ctx.set_narrow_kernel(k)
     outs.append(ctx.bootstrap_wo_ks(ct))
 ctx.set_narrow_kernel(0)
