@@ -1,3 +1,6 @@
+# A/B of an L2 persistence window over the BK (r02p2).  TB_BK_PERSIST was read only by the experimental build
+# (run_br set cudaStreamAttributeAccessPolicyWindow around the br6 launch); that code was not kept, see
+# profiles/r02p2_bk_l2_persist_ab.txt and DESIGN.md 7.1.
 O=gpurun_out
 for r in ${RATIOS:-0 0.5 1.0}; do
   if [ "$r" = "0" ]; then unset TB_BK_PERSIST; else export TB_BK_PERSIST=$r; fi
