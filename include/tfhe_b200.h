@@ -84,7 +84,8 @@ int tb_gates(tb_ctx* ctx, int gate, const uint32_t* ca, const uint32_t* cb, cons
              uint32_t* out, int64_t count, int64_t stride, tb_stream stream);
 
 /* Same, HOST arrays (end-to-end path: host->device copies, gates, device->host copy, synchronise).  Uses
- * context-owned device staging buffers. */
+ * context-owned device staging buffers.  On any error the call still returns only after every copy it queued
+ * from / into the host arrays has finished. */
 int tb_gates_host(tb_ctx* ctx, int gate, const uint32_t* host_ca, const uint32_t* host_cb,
                   const uint32_t* host_cc, uint32_t* host_out, int64_t count, int64_t stride);
 
@@ -159,7 +160,8 @@ int tb_run_netlist(tb_ctx* ctx, const tb_dev_netlist* dnet, uint32_t* wires, int
  * the n_outputs wires listed in output_wires (original wire ids, host array) to host_outputs (rows of
  * out_stride >= 631 words).  The input copies run on their own stream in the order of the level that first reads
  * them (level L waits only for its inputs) and the outputs of level L are copied back while level L + 1 runs
- * (SURVEY 8(f) f1); pinned host buffers make the copies asynchronous.  Synchronous. */
+ * (SURVEY 8(f) f1); pinned host buffers make the copies asynchronous.  Synchronous, also on error (no copy
+ * from / into the host buffers is in flight when it returns). */
 int tb_run_netlist_host(tb_ctx* ctx, const tb_dev_netlist* dnet, const uint32_t* host_inputs, int64_t in_stride,
                         const int64_t* output_wires, int64_t n_outputs, uint32_t* host_outputs, int64_t out_stride);
 /* tb_run_netlist_host: overlap the copies with the level loop (1, default) or run copy, levels, copy back one

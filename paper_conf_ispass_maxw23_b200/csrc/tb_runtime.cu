@@ -591,8 +591,19 @@ extern "C" int tb_gates(tb_ctx* c, int gate, const uint32_t* ca, const uint32_t*
     return run_ks(c, c->lanebuf, 0, kLaneStride, c->gdesc, count, out, stride, ca, stride, st);
 }
 
+static int gates_host_impl(tb_ctx* c, int gate, const uint32_t* hca, const uint32_t* hcb, const uint32_t* hcc,
+                           uint32_t* hout, int64_t count, int64_t stride);
 extern "C" int tb_gates_host(tb_ctx* c, int gate, const uint32_t* hca, const uint32_t* hcb, const uint32_t* hcc,
                              uint32_t* hout, int64_t count, int64_t stride) {
+    const int rc = gates_host_impl(c, gate, hca, hcb, hcc, hout, count, stride);
+    if (rc != TB_OK && c && c->own) {   // no copy from / into the caller's host buffers may still be in flight
+        cudaStreamSynchronize(c->own);
+        cudaGetLastError();
+    }
+    return rc;
+}
+static int gates_host_impl(tb_ctx* c, int gate, const uint32_t* hca, const uint32_t* hcb, const uint32_t* hcc,
+                           uint32_t* hout, int64_t count, int64_t stride) {
     int rc = check_ready(c);
     if (rc) return rc;
     if (count < 0 || stride < kn + 1) return fail(TB_EINVAL, "bad count or stride");
@@ -1234,8 +1245,20 @@ extern "C" int tb_set_host_overlap(tb_ctx* c, int enable) {
 // work of another).  The input rows are copied on their own stream in the order of the level that first reads
 // them, and level L waits only for the inputs it reads; the requested outputs produced by level L are copied back
 // on a second stream while level L + 1 runs.  With overlap off (tb_set_host_overlap(0)) everything is serial.
+static int run_netlist_host_impl(tb_ctx* c, const tb_dev_netlist* d, const uint32_t* hin, int64_t in_stride,
+                                 const int64_t* outw, int64_t n_out, uint32_t* hout, int64_t out_stride);
 extern "C" int tb_run_netlist_host(tb_ctx* c, const tb_dev_netlist* d, const uint32_t* hin, int64_t in_stride,
                                    const int64_t* outw, int64_t n_out, uint32_t* hout, int64_t out_stride) {
+    const int rc = run_netlist_host_impl(c, d, hin, in_stride, outw, n_out, hout, out_stride);
+    if (rc != TB_OK && c) {   // no copy from / into the caller's host buffers may still be in flight on return
+        for (cudaStream_t s : {c->own, c->h2d, c->d2h})
+            if (s) cudaStreamSynchronize(s);
+        cudaGetLastError();
+    }
+    return rc;
+}
+static int run_netlist_host_impl(tb_ctx* c, const tb_dev_netlist* d, const uint32_t* hin, int64_t in_stride,
+                                 const int64_t* outw, int64_t n_out, uint32_t* hout, int64_t out_stride) {
     int rc = check_ready(c);
     if (rc) return rc;
     if (!d || (d->n_inputs > 0 && !hin) || (n_out > 0 && (!outw || !hout))) return fail(TB_EINVAL, "null argument");
