@@ -160,7 +160,9 @@ int tb_run_netlist(tb_ctx* ctx, const tb_dev_netlist* dnet, uint32_t* wires, int
  * the n_outputs wires listed in output_wires (original wire ids, host array) to host_outputs (rows of
  * out_stride >= 631 words).  The input copies run on their own stream in the order of the level that first reads
  * them (level L waits only for its inputs) and the outputs of level L are copied back while level L + 1 runs
- * (SURVEY 8(f) f1); pinned host buffers make the copies asynchronous.  Synchronous, also on error (no copy
+ * (SURVEY 8(f) f1); a level of more than 8 waves of the throughput kernel (a wave = 4 x SM-count gates) runs as
+ * three launches (3 waves, the middle, the last 3-4 waves) so that the copies overlap inside a wide level too.
+ * Pinned host buffers make the copies asynchronous.  Synchronous, also on error (no copy
  * from / into the host buffers is in flight when it returns). */
 int tb_run_netlist_host(tb_ctx* ctx, const tb_dev_netlist* dnet, const uint32_t* host_inputs, int64_t in_stride,
                         const int64_t* output_wires, int64_t n_outputs, uint32_t* host_outputs, int64_t out_stride);

@@ -143,6 +143,7 @@ struct tb_dev_netlist {
     std::vector<int64_t> row_of_wire;       // [n_inputs + n_gates]
     int world = 1;                          // ranks the level order was planned for
     std::vector<int64_t> in_level;          // [n_inputs] first level that reads the input (n_levels + 1: none)
+    std::vector<int64_t> in_first;          // [n_inputs] first level-sorted gate position reading it (n_gates: none)
     std::vector<int64_t> early;             // [n_levels][world]: gates at the start of rank r's chunk of a level
                                             // whose inputs are local once r has run its part of the level before
     LaneDesc* ldesc = nullptr;
@@ -1008,13 +1009,17 @@ extern "C" int tb_netlist_upload(tb_ctx* c, const tb_netlist* net, tb_dev_netlis
     const int64_t ni = net->n_inputs, ng = net->n_gates;
     d->n_inputs = ni; d->n_gates = ng;
     d->in_level.assign((size_t)ni, d->n_levels + 1);
+    d->in_first.assign((size_t)ni, ng);
     for (int64_t L = 1; L <= d->n_levels; L++)
         for (int64_t k = d->level_off[L - 1]; k < d->level_off[L]; k++) {
             const int64_t g = order[k];
             const int t = net->type[g];
             const int64_t w[3] = {net->in0[g], t == TB_NOT ? -1 : net->in1[g], t == TB_MUX ? net->in2[g] : -1};
             for (int64_t x : w)
-                if (x >= 0 && x < ni) d->in_level[x] = std::min(d->in_level[x], L);
+                if (x >= 0 && x < ni) {
+                    d->in_level[x] = std::min(d->in_level[x], L);
+                    d->in_first[x] = std::min(d->in_first[x], k);
+                }
         }
     // descriptors in level-sorted order
     std::vector<GateDesc> gd((size_t)ng);
@@ -1247,6 +1252,9 @@ extern "C" int tb_set_host_overlap(tb_ctx* c, int enable) {
 // on a second stream while level L + 1 runs.  With overlap off (tb_set_host_overlap(0)) everything is serial.
 static int run_netlist_host_impl(tb_ctx* c, const tb_dev_netlist* d, const uint32_t* hin, int64_t in_stride,
                                  const int64_t* outw, int64_t n_out, uint32_t* hout, int64_t out_stride);
+// tb_run_netlist_host: a level of more than kHostChunkMinWaves waves of br6 (4 lanes per SM) runs as a first and a
+// last chunk of kHostEdgeWaves waves around the rest, so that the copies overlap inside a wide level as well
+constexpr int64_t kHostChunkMinWaves = 8, kHostEdgeWaves = 3;
 extern "C" int tb_run_netlist_host(tb_ctx* c, const tb_dev_netlist* d, const uint32_t* hin, int64_t in_stride,
                                    const int64_t* outw, int64_t n_out, uint32_t* hout, int64_t out_stride) {
     const int rc = run_netlist_host_impl(c, d, hin, in_stride, outw, n_out, hout, out_stride);
@@ -1286,47 +1294,71 @@ static int run_netlist_host_impl(tb_ctx* c, const tb_dev_netlist* d, const uint3
     if (ov && !c->h2d) TB_CUDA(cudaStreamCreateWithFlags(&c->h2d, cudaStreamNonBlocking));
     if (ov && !c->d2h) TB_CUDA(cudaStreamCreateWithFlags(&c->d2h, cudaStreamNonBlocking));
     cudaStream_t cs = c->own, hs = ov ? c->h2d : c->own, ds = ov ? c->d2h : c->own;
-    const size_t nev = 2 * (size_t)(nL + 2);
+    // ---- chunks: a level of more than 8 waves of the throughput kernel (W = 4 lanes x SM count) runs as three
+    // launches -- 3 W, the middle (a multiple of W, so no wave is added), the rest (3 W .. 4 W) -- so that the
+    // copies overlap inside a wide level too: the middle's inputs land while the first chunk runs, the middle's
+    // outputs leave while the last chunk runs; only the first chunk's inputs and the last chunk's outputs are
+    // exposed.  (Chunks of 16 W throughout were measured slower: each key-switch launch has its own tail.)
+    if (c->sms == 0 && cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess)
+        c->sms = 148;
+    const int64_t W = 4 * (int64_t)c->sms;
+    std::vector<int64_t> bnd{0};                      // chunk boundaries in level-sorted gate positions
+    std::vector<int64_t> lvl_of_chunk;
+    for (int64_t L = 1; L <= nL; L++) {
+        const int64_t a0 = d->level_off[L - 1], a1 = d->level_off[L], n = a1 - a0;
+        if (ov && n > kHostChunkMinWaves * W) {
+            const int64_t mid = (n - 2 * kHostEdgeWaves * W) / W * W;
+            for (int64_t e : {a0 + kHostEdgeWaves * W, a0 + kHostEdgeWaves * W + mid, a1}) {
+                bnd.push_back(e);
+                lvl_of_chunk.push_back(L);
+            }
+        } else if (n > 0) {
+            bnd.push_back(a1);
+            lvl_of_chunk.push_back(L);
+        }
+    }
+    const int64_t nC = (int64_t)lvl_of_chunk.size();
+    auto chunk_of = [&](int64_t k) {                  // chunk of gate position k (nC: none)
+        return (int64_t)(std::upper_bound(bnd.begin(), bnd.end(), k) - bnd.begin()) - 1;
+    };
+    const size_t nev = 2 * (size_t)(nC + 2);
     while (c->hev.size() < nev) {
         cudaEvent_t e;
         TB_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
         c->hev.push_back(e);
     }
-    auto ev_in = [&](int64_t L) { return c->hev[(size_t)L]; };             // inputs of level L landed
-    auto ev_out = [&](int64_t L) { return c->hev[(size_t)(nL + 2 + L)]; }; // level L's outputs are final
-    // ---- inputs: runs of consecutive rows with the same first level, in level order
-    std::vector<int64_t> by_level;                    // input rows sorted by (first level, row)
-    by_level.resize((size_t)d->n_inputs);
-    for (int64_t w = 0; w < d->n_inputs; w++) by_level[w] = w;
-    std::stable_sort(by_level.begin(), by_level.end(),
-                     [&](int64_t x, int64_t y) { return d->in_level[x] < d->in_level[y]; });
-    std::vector<char> has_in((size_t)nL + 2, 0);
-    for (size_t a = 0; a < by_level.size();) {
-        const int64_t L = d->in_level[by_level[a]];
+    auto ev_in = [&](int64_t j) { return c->hev[(size_t)j]; };             // inputs of chunk j landed
+    auto ev_out = [&](int64_t j) { return c->hev[(size_t)(nC + 2 + j)]; }; // chunk j's outputs are final
+    // ---- inputs: runs of consecutive rows with the same first chunk, in chunk order
+    std::vector<int64_t> in_chunk((size_t)d->n_inputs), by_chunk((size_t)d->n_inputs);
+    for (int64_t w = 0; w < d->n_inputs; w++) {
+        in_chunk[(size_t)w] = d->in_first[w] >= d->n_gates ? nC : chunk_of(d->in_first[w]);
+        by_chunk[(size_t)w] = w;
+    }
+    if (!std::is_sorted(in_chunk.begin(), in_chunk.end()))     // (already in chunk order: the common layout)
+        std::stable_sort(by_chunk.begin(), by_chunk.end(),
+                         [&](int64_t x, int64_t y) { return in_chunk[(size_t)x] < in_chunk[(size_t)y]; });
+    std::vector<char> has_in((size_t)nC + 1, 0);
+    for (size_t a = 0; a < by_chunk.size();) {
+        const int64_t j = in_chunk[(size_t)by_chunk[a]];
         size_t b = a + 1;
-        while (b < by_level.size() && d->in_level[by_level[b]] == L && by_level[b] == by_level[b - 1] + 1) b++;
-        TB_CUDA(cudaMemcpy2DAsync(c->hwires + (size_t)by_level[a] * S, S * 4, hin + (size_t)by_level[a] * in_stride,
+        while (b < by_chunk.size() && in_chunk[(size_t)by_chunk[b]] == j && by_chunk[b] == by_chunk[b - 1] + 1) b++;
+        TB_CUDA(cudaMemcpy2DAsync(c->hwires + (size_t)by_chunk[a] * S, S * 4, hin + (size_t)by_chunk[a] * in_stride,
                                   in_stride * 4, (kn + 1) * 4, b - a, cudaMemcpyHostToDevice, hs));
-        const bool last_of_level = b == by_level.size() || d->in_level[by_level[b]] != L;
-        if (last_of_level) {
-            TB_CUDA(cudaEventRecord(ev_in(std::min(L, nL + 1)), hs));
-            has_in[(size_t)std::min(L, nL + 1)] = 1;
+        if (b == by_chunk.size() || in_chunk[(size_t)by_chunk[b]] != j) {
+            TB_CUDA(cudaEventRecord(ev_in(j), hs));
+            has_in[(size_t)j] = 1;
         }
         a = b;
     }
-    // ---- outputs grouped by the level that produces them (0: an input passed through)
-    std::vector<int64_t> lvl_of_row;                  // level of a gate row
-    std::vector<std::vector<int64_t>> outs_at((size_t)nL + 1);
+    // ---- outputs grouped by the chunk that produces them (index nC: an input passed through)
+    std::vector<std::vector<int64_t>> outs_at((size_t)nC + 1);
     for (int64_t k = 0; k < n_out; k++) {
         const int64_t r = rows[k];
-        int64_t L = 0;
-        if (r >= d->n_inputs)
-            L = (int64_t)(std::upper_bound(d->level_off.begin(), d->level_off.end(), r - d->n_inputs) -
-                          d->level_off.begin());
-        outs_at[(size_t)L].push_back(k);
+        outs_at[(size_t)(r >= d->n_inputs ? chunk_of(r - d->n_inputs) : nC)].push_back(k);
     }
-    auto copy_outs = [&](int64_t L) -> int {
-        const auto& ks = outs_at[(size_t)L];
+    auto copy_outs = [&](int64_t j) -> int {
+        const auto& ks = outs_at[(size_t)j];
         for (size_t a = 0; a < ks.size();) {
             size_t b = a + 1;
             while (b < ks.size() && ks[b] == ks[b - 1] + 1 && rows[ks[b]] == rows[ks[b - 1]] + 1) b++;
@@ -1337,21 +1369,22 @@ static int run_netlist_host_impl(tb_ctx* c, const tb_dev_netlist* d, const uint3
         }
         return TB_OK;
     };
-    // ---- the level loop on the compute stream
-    for (int64_t L = 1; L <= nL; L++) {
-        if (has_in[(size_t)L]) TB_CUDA(cudaStreamWaitEvent(cs, ev_in(L), 0));
-        const int64_t n = d->level_off[L] - d->level_off[L - 1];
-        if ((rc = tb_run_level(c, d, L, 0, n, c->hwires, S, (tb_stream)cs))) return rc;
-        if (!outs_at[(size_t)L].empty()) {
-            TB_CUDA(cudaEventRecord(ev_out(L), cs));
-            TB_CUDA(cudaStreamWaitEvent(ds, ev_out(L), 0));
-            if ((rc = copy_outs(L))) return rc;
+    // ---- the level loop on the compute stream, chunk by chunk
+    for (int64_t j = 0; j < nC; j++) {
+        if (has_in[(size_t)j]) TB_CUDA(cudaStreamWaitEvent(cs, ev_in(j), 0));
+        const int64_t L = lvl_of_chunk[(size_t)j], a0 = d->level_off[L - 1];
+        if ((rc = tb_run_level(c, d, L, bnd[(size_t)j] - a0, bnd[(size_t)j + 1] - a0, c->hwires, S, (tb_stream)cs)))
+            return rc;
+        if (!outs_at[(size_t)j].empty()) {
+            TB_CUDA(cudaEventRecord(ev_out(j), cs));
+            TB_CUDA(cudaStreamWaitEvent(ds, ev_out(j), 0));
+            if ((rc = copy_outs(j))) return rc;
         }
     }
-    if (!outs_at[0].empty()) {                        // outputs that are inputs: after every input copy
-        for (int64_t L = 1; L <= nL + 1; L++)
-            if (has_in[(size_t)L]) TB_CUDA(cudaStreamWaitEvent(ds, ev_in(L), 0));
-        if ((rc = copy_outs(0))) return rc;
+    if (!outs_at[(size_t)nC].empty()) {               // outputs that are inputs: after every input copy
+        for (int64_t j = 0; j <= nC; j++)
+            if (has_in[(size_t)j]) TB_CUDA(cudaStreamWaitEvent(ds, ev_in(j), 0));
+        if ((rc = copy_outs(nC))) return rc;
     }
     TB_CUDA(cudaStreamSynchronize(hs));
     TB_CUDA(cudaStreamSynchronize(cs));

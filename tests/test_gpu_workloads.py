@@ -150,6 +150,44 @@ def test_run_netlist_host_overlap_equals_serial(tb, ctx, keys):
         assert (o == ref[ow]).all()
 
 
+def test_run_netlist_host_chunked_wide_level(tb, ctx, keys):
+    """tb_run_netlist_host runs a level of more than 8 waves of br6 (a wave = 4 x SM-count gates) as three chunks
+    (3 waves, the middle, the rest) whose input copies land, and whose outputs leave, while the neighbouring
+    chunks run: a 20,000-gate level followed by gates that read across both chunk boundaries gives the same bytes
+    as the device path, overlapped and serial, and the second-level results decrypt to the plaintext"""
+    import torch
+    G1 = 20000
+    W = 4 * torch.cuda.get_device_properties(0).multi_processor_count
+    b1 = 3 * W
+    b2 = b1 + (G1 - 6 * W) // W * W
+    lv = synth.independent_level(G1, 17)
+    ni = lv["n_inputs"]
+    w = lambda g: ni + g                                            # wire of level-1 gate g
+    pairs = [(0, G1 - 1), (b1 - 1, b1), (b2 - 1, b2), (100, b2 + 5), (G1 - 2, 5)]
+    t2 = np.array([synth.XOR, synth.XOR, synth.AND, synth.AND, synth.OR], np.int32)
+    n = dict(n_inputs=ni, type=np.concatenate([lv["type"], t2]),
+             in0=np.concatenate([lv["in0"], [w(a) for a, _ in pairs]]).astype(np.int64),
+             in1=np.concatenate([lv["in1"], [w(b) for _, b in pairs]]).astype(np.int64),
+             in2=np.full(G1 + len(pairs), -1, np.int64))
+    n["outputs"] = np.arange(ni + G1, ni + G1 + len(pairs), dtype=np.int64)
+    bits = synth.random_bits(ni, 18)
+    cts = O.encrypt_bits(keys, bits, 19)
+    ref, dnet = run(tb, ctx, n, cts)
+    ow = np.concatenate([n["outputs"], np.arange(ni + G1 - 1, 0, -997)]).astype(np.int64)   # + sampled wires
+    for overlap in (True, False):
+        ctx.set_host_overlap(overlap)
+        try:
+            got = ctx.run_netlist_host(dnet, cts, ow)
+        finally:
+            ctx.set_host_overlap(True)
+        assert (got == ref[ow]).all(), overlap
+    f = {synth.NAND: lambda a, b: 1 - (a & b), synth.XOR: lambda a, b: a ^ b, synth.AND: lambda a, b: a & b,
+         synth.OR: lambda a, b: a | b}
+    l1 = np.array([f[int(t)](int(bits[2 * g]), int(bits[2 * g + 1])) for g, t in enumerate(lv["type"])])
+    want = [f[int(t)](int(l1[a]), int(l1[b])) for t, (a, b) in zip(t2, pairs)]
+    assert O.decrypt_bits(keys, got[:len(pairs)]).tolist() == want
+
+
 def test_same_wire_twice_and_duplicate_consumers(tb, ctx, keys):
     """XOR(a, a) = 0 and AND(a, a) = a; one wire feeding many gates of a level"""
     n = dict(n_inputs=2, type=np.array([6, 8, 7, 7, 14], np.int32), in0=np.array([0, 0, 0, 1, 2]),
