@@ -68,8 +68,9 @@ int tb_ctx_destroy(tb_ctx* ctx);
 
 /* Bootstrapping key, HOST pointer, torus layout [i < n][row r = bloc*l + j < 2l][poly < 2][N] u32
  * (n_words must equal n*2l*2*N = 7,741,440).  The torus key stays on the device (31 MB) and only the transform
- * domains that the selected kernels read are built from it: the NTT domain (br6 / br9: each coefficient split
- * into 3 signed parts, 92.9 MB), the FFT domain (brf / brl, 123.9 MB), the four-step NTT domain (brt, 92.9 MB).
+ * domains that the selected kernels read are built from it: the NTT domain (br6 / br6t / br9: each coefficient
+ * split into 3 signed parts, 92.9 MB), the FFT domain (brf / brl / brl2, 123.9 MB), the four-step NTT domain
+ * (brt / brq / brtl, 92.9 MB).
  * Selecting another kernel later (tb_set_br_variant / tb_set_narrow_kernel / tb_set_narrow_lanes) builds the
  * domains it needs then (synchronously).  No host copy is kept.  Synchronous. */
 int tb_load_bk(tb_ctx* ctx, const uint32_t* host_bk, size_t n_words);
@@ -207,12 +208,13 @@ int tb_set_br_variant(tb_ctx* ctx, int variant);
 /* Latency mode for narrow levels: a launch with <= `lanes` bootstraps runs a latency-mode kernel (below)
  * instead of the throughput kernel.  Default = the device's SM count; 0 disables. */
 int tb_set_narrow_lanes(tb_ctx* ctx, int64_t lanes);
-/* Latency-mode kernel: 0 = auto (default: brl while the level's bootstraps fit in one wave of brl clusters, br9
- * while they fit one wave of its SM pairs, else brtl), 11 = brl_kernel (one bootstrap per cluster of 4 SMs on the
- * FP64 path: each SM owns one output polynomial and one 16-bit BK half; 1.9 ms per level on B200, 32 per wave),
- * 9 = br9_kernel (one bootstrap per cluster of 2 SMs, forward-NTT rows exchanged through distributed shared memory;
- * 3.5 ms, 74 per wave), 13 = brtl_kernel (one bootstrap per SM on the tensor cores, tb_brtl.cu; 4.7 ms, 148 per
- * wave).  All are bit-identical.  Anything else: TB_EINVAL. */
+/* Latency-mode kernel: 0 = auto (default: brl while the level's bootstraps fit in one wave of brl clusters, else
+ * brl2), 11 = brl_kernel (one bootstrap per cluster of 4 SMs on the FP64 path: each SM owns one output polynomial
+ * and one 16-bit BK half; 1.9 ms per level on B200, 32 per wave), 16 = brl2_kernel (one bootstrap per cluster of 2
+ * SMs on the FP64 path: each SM owns one output polynomial and both BK halves, tb_brl2.cu; 2.1 ms, 74 per wave),
+ * 9 = br9_kernel (one bootstrap per cluster of 2 SMs, integer NTT, forward-NTT rows exchanged through distributed
+ * shared memory; 3.5 ms, 74 per wave), 13 = brtl_kernel (one bootstrap per SM on the tensor cores, tb_brtl.cu;
+ * 4.7 ms, 148 per wave).  All are bit-identical.  Anything else: TB_EINVAL. */
 int tb_set_narrow_kernel(tb_ctx* ctx, int kernel);
 /* Level schedule used by tb_netlist_upload: Algorithm 1 gives every gate its earliest level;
  * with lanes > 0 gates that have slack are moved to later levels (never past their latest level, so the number

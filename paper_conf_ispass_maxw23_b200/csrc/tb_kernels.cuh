@@ -88,6 +88,9 @@ namespace tb {
 int launch_brf(const BrArgs& A, int G, const double2* bkf, const double2* twB, const double2* twC, cudaStream_t st);
 void launch_bk_to_fft(const uint32_t* bk, double2* bkf, const double2* twB, const double2* twC, cudaStream_t st);
 size_t bkf_bytes();
+// latency mode, one bootstrap per 2-SM cluster on the FP64 pipe (tb_brl2.cu); brl2_wave_lanes = co-resident clusters
+int launch_brl2(const BrArgs& A, const double2* bkf, const double2* twL, cudaStream_t st);
+int brl2_wave_lanes();
 int launch_brl(const BrArgs& A, const double2* bkf, const double2* twL, cudaStream_t st);
 int brl_wave_lanes();
 }  // namespace tb

@@ -64,9 +64,10 @@ struct tb_ctx {
     int variant = 6;                        // blind-rotation kernel: 6 = br6, 10 = brf (FP64 pipe)
     int ks_tile = 8;                        // gates per key-switch CTA (8, 16, 32); 8 measured fastest
     int narrow_lanes = 0;                   // launches with <= this many lanes run in latency mode (= SM count)
-    int narrow_kernel = 0;                  // latency-mode kernel: 9 = br9 (2-SM cluster per lane),
-                                            // 11 = brl (4-SM cluster per lane, FP64 path), 0 = auto:
-                                            // brl while the lanes fit in one wave of its clusters, else br9
+    int narrow_kernel = 0;                  // latency-mode kernel: 9 = br9 (2-SM cluster per lane), 11 = brl
+                                            // (4-SM cluster per lane, FP64 path), 13 = brtl (one SM per lane,
+                                            // tensor cores), 16 = brl2 (2-SM cluster per lane, FP64 path),
+                                            // 0 = auto: brl while the lanes fit one wave of its clusters, else brl2
     int brl_wave = -2;                      // co-resident brl clusters (queried on first use)
     int plan_world = 1;                     // netlist upload: order each level for this many ranks (early gates first)
     int64_t level_capacity = -1;            // netlist upload: re-levelise to <= this many lanes per level where
@@ -355,7 +356,8 @@ static unsigned needed_domains(const tb_ctx* c) {
         if (c->narrow_kernel == 9) m |= kDomNtt;
         else if (c->narrow_kernel == 11) m |= kDomFft;
         else if (c->narrow_kernel == 13) m |= kDomBk4;
-        else m |= kDomNtt | kDomFft | kDomBk4;         // auto: brl, br9 or brtl by the level's width
+        else if (c->narrow_kernel == 16) m |= kDomFft;
+        else m |= kDomFft;                             // auto: brl or brl2 by the level's width
     }
     return m;
 }
@@ -384,8 +386,8 @@ extern "C" int tb_set_br_variant(tb_ctx* c, int variant) {
 }
 
 extern "C" int tb_set_narrow_kernel(tb_ctx* c, int kernel) {
-    if (!c || (kernel != 0 && kernel != 9 && kernel != 11 && kernel != 13))
-        return fail(TB_EINVAL, "latency-mode kernel must be 0 (auto), 9, 11 or 13");
+    if (!c || (kernel != 0 && kernel != 9 && kernel != 11 && kernel != 13 && kernel != 16))
+        return fail(TB_EINVAL, "latency-mode kernel must be 0 (auto), 9, 11, 13 or 16");
     c->narrow_kernel = kernel;
     return build_domains(c);
 }
@@ -509,15 +511,15 @@ static int run_br(tb_ctx* c, const uint32_t* s0, const uint32_t* s1, const uint3
     const long slot = prof_begin(c, 0, st);
     int rc;
     int nk = c->narrow_kernel;
-    if (nk == 0) {   // auto (profiles/r02y_latency.jsonl): brl while the lanes fit its 32 clusters (1.9 ms), br9
-                     // while they fit its SM pairs (3.5 ms), beyond that brtl with one lane per SM (4.7 ms flat)
+    if (nk == 0) {   // auto (profiles/r02l2_latency.jsonl): brl while the lanes fit its 32 four-SM clusters
+                     // (1.9-2.0 ms), beyond that brl2 on SM pairs (2.1 ms up to 74 lanes, 4.2 ms up to 148; br9 was
+                     // 3.5 / 7.1 ms there and brtl 4.7 ms)
         if (c->brl_wave == -2) c->brl_wave = brl_wave_lanes();
-        if (c->sms == 0 && cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess)
-            c->sms = 148;
-        nk = nlanes <= c->brl_wave ? 11 : (nlanes <= c->sms / 2 ? 9 : 13);
+        nk = nlanes <= c->brl_wave ? 11 : 16;
     }
     if (c->narrow_lanes > 0 && nlanes <= c->narrow_lanes)
         rc = nk == 9    ? launch_br9(A, st)                    // narrow level: one lane per 2-SM cluster
+             : nk == 16 ? launch_brl2(A, c->bkf, c->fftL, st)  // or per 2-SM cluster (FP64)
              : nk == 13 ? launch_brtl(A, c->bk4, c->tcB, c->tcTw, st)   // or per SM on the tensor cores
                         : launch_brl(A, c->bkf, c->fftL, st);  // or per 4-SM cluster (FP64)
     else if (c->variant == 12)

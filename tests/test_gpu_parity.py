@@ -96,19 +96,21 @@ def oracle_bootstrap_many(keys, cts):
         return np.stack(list(ex.map(lambda c: O.bootstrap_wo_ks(keys, c), cts)))
 
 
-@pytest.mark.parametrize("kernel", [0, 9, 11, 13])
+@pytest.mark.parametrize("kernel", [0, 9, 11, 13, 16])
 def test_narrow_level_latency_mode_bit_exact(tb, ctx, keys, kernel):
     """small launches run the latency kernel (br9: 2-SM cluster per lane, brl: 4-SM cluster per lane on the
-    FP64 path, brtl: one SM per lane on the tensor cores; 40 lanes = 160 CTAs is more than one wave of brl);
-    149 lanes fall back to the throughput kernel.
-    Every lane of the 1-, 3- and 40-lane launches is compared with the oracle, the first and last of 149."""
+    FP64 path, brtl: one SM per lane on the tensor cores, brl2: 2-SM cluster per lane on the FP64 path; 40 lanes =
+    160 CTAs is more than one wave of brl, 80 lanes more than one wave of brl2 / br9); 149 lanes fall back to the
+    throughput kernel.  Every lane of the 1-, 3- and 40-lane launches is compared with the oracle, three of 80
+    (first, one in the second wave, last) and the first and last of 149."""
     rng = np.random.default_rng(39 + kernel)
     ctx.set_narrow_kernel(kernel)
     try:
-        for count in (1, 3, 40, 149):
+        for count in (1, 3, 40, 80, 149):
             cts = rng.integers(0, M32, (count, 631), dtype=np.uint64).astype(np.uint32)
             got = ctx.bootstrap_wo_ks(ctx.to_device(cts))[:, :1025].cpu().numpy().view(np.uint32)
-            idx = np.arange(count) if count <= 40 else np.array([0, count - 1])
+            idx = np.arange(count) if count <= 40 else (np.array([0, 77, count - 1]) if count == 80
+                                                         else np.array([0, count - 1]))
             assert (got[idx] == oracle_bootstrap_many(keys, cts[idx])).all(), count
     finally:
         ctx.set_narrow_kernel(0)

@@ -24,8 +24,9 @@ def main():
         if k == 6:
             ctx.set_narrow_lanes(0)
         else:
+            ctx.set_narrow_lanes(1000)                     # latency mode for every width measured here
             ctx.set_narrow_kernel(k)
-        for lanes in (1, 4, 16, 32, 37, 74, 100, 148) + ((200, 296, 400, 592) if k == 6 else ()):
+        for lanes in (1, 4, 16, 32, 37, 74, 100, 148) + ((200, 222, 296, 400, 592) if k in (6, 16) else ()):
             a, b = ctx.empty(lanes), ctx.empty(lanes)
             a.random_(-2 ** 31, 2 ** 31 - 1, generator=g)
             b.random_(-2 ** 31, 2 ** 31 - 1, generator=g)

@@ -45,11 +45,11 @@ if BRT:
 if LAT:
     one = ct[:1]
     res = []
-    for k in (11, 9):
+    for k in (11, 9, 16):
         ctx.set_narrow_kernel(k)
         res.append(ctx.bootstrap_wo_ks(one))
     torch.cuda.synchronize()
-    ok = torch.equal(res[0][:, :1025], res[1][:, :1025])
+    ok = all(torch.equal(res[0][:, :1025], r[:, :1025]) for r in res[1:])
     print("latency kernels agree:", ok)
     sys.exit(0 if ok else 1)
 NOBRT = os.environ.get("TB_SAN_NOBRT") == "1"                # synccheck: the tool does not model tcgen05.commit
@@ -59,7 +59,7 @@ for variant in ((6,) if QUICK else ((6, 10) if NOBRT else (6, 10, 12, 14, 15))):
     outs.append(ctx.bootstrap_wo_ks(ct))
 ctx.set_br_variant(6)
 ctx.set_narrow_lanes(148)
-for k in (() if QUICK else ((11, 9) if NOBRT else (11, 9, 13))):   # latency mode: brl, br9, brtl
+for k in (() if QUICK else ((11, 9, 16) if NOBRT else (11, 9, 13, 16))):   # latency: brl, br9, brtl, brl2
     ctx.set_narrow_kernel(k)
     outs.append(ctx.bootstrap_wo_ks(ct))
 ctx.set_narrow_kernel(0)
