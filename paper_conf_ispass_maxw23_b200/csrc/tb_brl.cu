@@ -22,6 +22,10 @@ namespace tb {
 
 constexpr int kLThreads = 256;                 // 8 warps: 3 forward transforms x 2 warps (0-5); warps 0-1 invert; all MAC
 constexpr int kLMacIt = (512 + kLThreads - 1) / kLThreads;
+#ifndef TB_BRL_BK_ISSUER
+#define TB_BRL_BK_ISSUER 64
+#endif
+constexpr int kBkIssuer = TB_BRL_BK_ISSUER;   // thread that issues the per-step BK TMA (outside warps 0-1)
 
 #ifdef TB_BRL_TRACE   // scratch instrumentation (tools/buildvar.sh WORK name -DTB_BRL_TRACE): clock64 per phase
 __device__ long long g_brl_trace[4][8][16];
@@ -311,7 +315,10 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         if ((tid & 63) == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // dslot rows sent
         __syncthreads();                                  // bk[buf], rrows[buf] consumed; oslot complete
         BRL_T(4)
-        if (tid == 0) {
+        // step i + 2's BK and the expectation of its rows: issued by a thread of warp 2, idle during the inverse
+        // (from warp 0, the fence.proxy.async + six bulk copies delayed the inverse's warp pair and the half
+        // swap behind it: one-gate level 1.92 -> 1.83 ms)
+        if (tid == kBkIssuer) {
             if (i + 2 < kn) {
                 mb_expect(&S.mbar_rows[buf], kL * 512 * 16);                  // rows of step i + 2
                 issue_bk_l(S, bkf, i + 2, o, buf);

@@ -43,6 +43,8 @@ __device__ __forceinline__ void issue_bk_l2(Brl2Smem& S, const double2* bkf, int
                 : "memory");
 }
 
+constexpr int kBk2Issuer = 128;   // issues the per-step BK TMA: warp 4 has no inverse to run
+
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
     brl2_kernel(BrArgs A, const double2* __restrict__ bkf, const double2* __restrict__ twL) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -164,7 +166,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
         }
         if ((tid & 63) == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // dslot rows sent
         __syncthreads();                                  // bk, rrows[buf] consumed; oslot complete
-        if (tid == 0) {
+        if (tid == kBk2Issuer) {   // a thread of warp 4, idle during the two inverses (warp pairs 0 and 1)
             if (i + 2 < kn) mb_expect(&S.mbar_rows[buf], kL * 512 * 16);   // rows of step i + 2
             if (i + 1 < kn) issue_bk_l2(S, bkf, i + 1, q);                  // lands during C and the next A
         }
