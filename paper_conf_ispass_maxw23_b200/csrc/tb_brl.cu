@@ -5,13 +5,16 @@
 // so the output is bit-identical to every other variant.  What changes is how one CMux step is spread out, to
 // shorten the serial chain of 630 steps that bounds a narrow netlist level:
 //   * CTA (q, h) of the cluster (rank 2q + h) owns output polynomial q and BK half h: it computes the 3 digit
-//     rows of ACC[q] (the two CTAs of a q compute them redundantly), sends them to CTA (1-q, h), runs the MAC
-//     for its one output o = 2q + h over all 6 rows, and one inverse transform; the two CTAs of a q swap their
-//     rounded halves and both add lo + 2^16 hi into their copy of ACC[q].
+//     rows of ACC[q] (the two CTAs of a q compute them redundantly) and splits the MAC by bloc (it is linear):
+//     its own rows times BK_i for its output o = 2q + h and for the partner CTA (1-q, h)'s output o2; it sends
+//     the o2 partial (8 KB; round 1 sent the three rows, 24 KB, and multiplied the received rows itself), adds
+//     the partner's partial of o, and runs one inverse transform; the two CTAs of a q swap their rounded halves
+//     and both add lo + 2^16 hi into their copy of ACC[q].  Summation order differs from the other variants,
+//     which the FP64 error bound does not depend on: the rounded products are identical.
 //   * every transform is split over 2 warps (64 threads x 8 values) and done as three radix-8 passes (stages
 //     1-3, 4-6, 7-9 of the merged-twist tree), with one shared-memory exchange between passes; the pass-2/3
 //     twiddles of a thread stay in registers for the whole kernel.
-//   * BK_i's 48 KB for output o are TMA-staged two steps ahead; rows and halves move CTA-to-CTA with
+//   * BK_i's 48 KB (own rows x outputs o, o2) are TMA-staged two steps ahead; partials and halves move CTA-to-CTA with
 //     shared::cluster bulk copies that complete on the receiver's mbarrier (double-buffered by step parity,
 //     safe for the same reason as br9's hand-over: a CTA can only send for step i+2 after it has received the
 //     receiver's data of step i+1, which the receiver produced after consuming step i).
@@ -26,6 +29,8 @@ constexpr int kLMacIt = (512 + kLThreads - 1) / kLThreads;
 #define TB_BRL_BK_ISSUER 64
 #endif
 constexpr int kBkIssuer = TB_BRL_BK_ISSUER;   // thread that issues the per-step BK TMA (outside warps 0-1)
+constexpr int kPsumPusher = 224;                // thread (warp 7) that pushes the partial
+constexpr uint32_t kRowsBytes = 512 * 16;   // the partner's partial MAC of this CTA's output (512 complex)
 
 #ifdef TB_BRL_TRACE   // scratch instrumentation (tools/buildvar.sh WORK name -DTB_BRL_TRACE): clock64 per phase
 __device__ long long g_brl_trace[4][8][16];
@@ -38,7 +43,8 @@ __device__ long long g_brl_trace[4][8][16];
 struct __align__(128) BrlSmem {
     double2 bk[2][kRows][512];                 // BK_i, rows 0..5 of output o = 2q + h, by step parity (96 KB)
     double2 dslot[kL][512];                    // own forward rows (bloc q), swizzled positions
-    double2 rrows[2][kL][512];                 // rows of bloc 1-q from CTA (1-q, h), by step parity
+    double2 psend[512];                        // partial MAC of the partner's output over the own rows
+    double2 precv[2][512];                     // the partner's partial MAC of this CTA's output, by step parity
     double2 oslot[512];                        // MAC output, then the inverse's exchange buffer
     uint32_t res[kN];                          // own rounded half of the product (sent to the sibling)
     uint32_t rres[2][kN];                      // the sibling's half, by step parity
@@ -172,17 +178,20 @@ __device__ __forceinline__ void push_peer(uint32_t dst, const void* src, uint32_
         : "memory");
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
-// BK_i rows 0..5 of output o -> bk[buf] (one thread)
-__device__ __forceinline__ void issue_bk_l(BrlSmem& S, const double2* bkf, int i, int o, int buf) {
+// BK_i -> bk[buf] (one thread): the own bloc's rows 3q..3q+2 of output o (slots 0-2) and of the partner's output
+// o2 (slots 3-5).
+__device__ __forceinline__ void issue_bk_l(BrlSmem& S, const double2* bkf, int i, int o, int o2, int q, int buf) {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     mb_expect(&S.mbar_bk[buf], kRows * 512 * 16);
 #pragma unroll
-    for (int r = 0; r < kRows; r++)
+    for (int r = 0; r < kRows; r++) {
+        const size_t row = (size_t)(i * kRows + kL * q + r % kL) * 4 + (r < kL ? o : o2);
         asm volatile(
             "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                 sm32(S.bk[buf][r])),
-            "l"(bkf + ((size_t)(i * kRows + r) * 4 + o) * 512), "r"(512 * 16), "r"(sm32(&S.mbar_bk[buf]))
+            "l"(bkf + row * 512), "r"(512 * 16), "r"(sm32(&S.mbar_bk[buf]))
             : "memory");
+    }
 }
 
 // twL: [64][6] per-thread pass bases: (pass 2: zeta_{4,t>>3}, zeta_{5,2(t>>3)}, zeta_{6,4(t>>3)},
@@ -194,6 +203,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint32_t rank = cl_rank();
     const int q = (int)(rank >> 1), h = (int)(rank & 1), o = 2 * q + h;
+    const int o2 = 2 * (1 - q) + h;                      // output of the partner CTA (1-q, h)
     const int gl = blockIdx.x >> 2;                      // one lane (bootstrap) per cluster
 
     if (tid == 0) {
@@ -204,14 +214,14 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         for (int b = 0; b < 2; b++) {                    // rows and halves of steps 0 and 1 may arrive any time
-            mb_expect(&S.mbar_rows[b], kL * 512 * 16);
+            mb_expect(&S.mbar_rows[b], kRowsBytes);
             mb_expect(&S.mbar_res[b], kN * 4);
         }
     }
     __syncthreads();
     if (tid == 0) {
-        issue_bk_l(S, bkf, 0, o, 0);
-        issue_bk_l(S, bkf, 1, o, 1);
+        issue_bk_l(S, bkf, 0, o, o2, q, 0);
+        issue_bk_l(S, bkf, 1, o, o2, q, 1);
     }
     {   // a1, a2 (every CTA of the cluster)
         LaneDesc d = {0, -1, 0, 0, 0u, 0u, 0u, 0u};
@@ -250,7 +260,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
     t3.a = ldc(twL + tt * 6 + 3);
     t3.b = ldc(twL + tt * 6 + 4);
     t3.c = ldc(twL + tt * 6 + 5);
-    const uint32_t rows_dst = cl_map(sm32(&S.rrows[0][0][0]), rank ^ 2u);
+    const uint32_t rows_dst = cl_map(sm32(&S.precv[0][0]), rank ^ 2u);
     const uint32_t rows_mb = cl_map(sm32(&S.mbar_rows[0]), rank ^ 2u);
     const uint32_t res_dst = cl_map(sm32(&S.rres[0][0]), rank ^ 1u);
     const uint32_t res_mb = cl_map(sm32(&S.mbar_res[0]), rank ^ 1u);
@@ -271,57 +281,56 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
                 x[v] = dcplx{small_to_double((u0 >> shift) & 127u, 64.0), small_to_double((u1 >> shift) & 127u, 64.0)};
             }
             fwd2w(x, S.dslot[jd], t1, t2, t3, tt, 1 + jd);
-            bar_pair(1 + jd);
-            if (tt == 0)   // row jd -> CTA (1-q, h) as soon as this warp pair is done
-                push_peer(rows_dst + (uint32_t)((buf * kL + jd) * 512 * 16), &S.dslot[jd][0], 512 * 16,
-                          rows_mb + (uint32_t)(buf * 8));
         }
         __syncthreads();
         BRL_T(1)
         mb_wait(&S.mbar_bk[buf], par);
         BRL_T(2)
-        // ---- B: out[k] = sum_{r<6} D_r[k] BK_i[r][o][k]; own bloc's rows first, then the other bloc's ----
+        // ---- B: the MAC split by bloc (it is linear): this CTA multiplies its own rows (bloc q) by BK_i for its
+        // output o and for the partner's output o2, sends the o2 partial (8 KB instead of 24 KB of rows), and adds
+        // the partner's partial of o.  Round-off: the FP64 error bound of §5b holds for any summation order. ----
         dcplx m3[kLMacIt];
 #pragma unroll
         for (int e = 0; e < kLMacIt; e++) {
             const int k = tid + kLThreads * e;
-            dcplx s = {0.0, 0.0};
+            dcplx s = {0.0, 0.0}, s2 = {0.0, 0.0};
             if (k < 512) {
 #pragma unroll
                 for (int r = 0; r < kL; r++) {
-                    const dcplx d = ldc(&S.dslot[r][lsw(k)]), b = ldc(&S.bk[buf][q * kL + r][k]);
+                    const dcplx d = ldc(&S.dslot[r][lsw(k)]);
+                    const dcplx b = ldc(&S.bk[buf][r][k]), b2 = ldc(&S.bk[buf][kL + r][k]);
                     s.re = fma(d.re, b.re, fma(-d.im, b.im, s.re));
                     s.im = fma(d.re, b.im, fma(d.im, b.re, s.im));
+                    s2.re = fma(d.re, b2.re, fma(-d.im, b2.im, s2.re));
+                    s2.im = fma(d.re, b2.im, fma(d.im, b2.re, s2.im));
                 }
+                stc(&S.psend[k], s2);
             }
             m3[e] = s;
         }
+        __syncthreads();                                  // psend complete
+        if (tid == kPsumPusher)
+            push_peer(rows_dst + (uint32_t)(buf * 512 * 16), S.psend, 512 * 16, rows_mb + (uint32_t)(buf * 8));
         mb_wait(&S.mbar_rows[buf], par);
         BRL_T(3)
 #pragma unroll
         for (int e = 0; e < kLMacIt; e++) {
             const int k = tid + kLThreads * e;
             if (k < 512) {
-                dcplx s = m3[e];
-#pragma unroll
-                for (int r = 0; r < kL; r++) {
-                    const dcplx d = ldc(&S.rrows[buf][r][lsw(k)]), b = ldc(&S.bk[buf][(1 - q) * kL + r][k]);
-                    s.re = fma(d.re, b.re, fma(-d.im, b.im, s.re));
-                    s.im = fma(d.re, b.im, fma(d.im, b.re, s.im));
-                }
-                stc(&S.oslot[lsw(k)], s);
+                const dcplx pr = ldc(&S.precv[buf][k]);
+                stc(&S.oslot[lsw(k)], dcplx{m3[e].re + pr.re, m3[e].im + pr.im});
             }
         }
-        if ((tid & 63) == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // dslot rows sent
-        __syncthreads();                                  // bk[buf], rrows[buf] consumed; oslot complete
+        if (tid == kPsumPusher) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // psend read
+        __syncthreads();                                  // bk[buf], precv[buf] consumed; oslot complete
         BRL_T(4)
         // step i + 2's BK and the expectation of its rows: issued by a thread of warp 2, idle during the inverse
         // (from warp 0, the fence.proxy.async + six bulk copies delayed the inverse's warp pair and the half
         // swap behind it: one-gate level 1.92 -> 1.83 ms)
         if (tid == kBkIssuer) {
             if (i + 2 < kn) {
-                mb_expect(&S.mbar_rows[buf], kL * 512 * 16);                  // rows of step i + 2
-                issue_bk_l(S, bkf, i + 2, o, buf);
+                mb_expect(&S.mbar_rows[buf], kRowsBytes);                     // rows / partial of step i + 2
+                issue_bk_l(S, bkf, i + 2, o, o2, q, buf);
             }
         }
         if (warp < 2) {   // ---- C: inverse (warp pair 0), round, << 16 h ----
