@@ -9,15 +9,17 @@
 //     its own rows times BK_i for its output o = 2q + h and for the partner CTA (1-q, h)'s output o2; it sends
 //     the o2 partial (8 KB; round 1 sent the three rows, 24 KB, and multiplied the received rows itself), adds
 //     the partner's partial of o, and runs one inverse transform; the two CTAs of a q swap their rounded halves
-//     and both add lo + 2^16 hi into their copy of ACC[q].  Summation order differs from the other variants,
-//     which the FP64 error bound does not depend on: the rounded products are identical.
+//     and both add lo + 2^16 hi into their copy of ACC[q].  The summation order differs from the other
+//     variants; the FP64 error bound does not depend on it, so the rounded products are identical.
+//   * both hand-overs are per-thread st.async stores straight from registers into the peer's shared memory,
+//     completing on its mbarrier (no staging buffer, no barrier and proxy fence before a bulk copy: one-gate
+//     level 1.79 -> 1.64 ms), double-buffered by step parity (safe for the same reason as br9's
+//     hand-over: a CTA can only send for step i+2 after it has received the receiver's data of step i+1, which
+//     the receiver produced after consuming step i).
 //   * every transform is split over 2 warps (64 threads x 8 values) and done as three radix-8 passes (stages
 //     1-3, 4-6, 7-9 of the merged-twist tree), with one shared-memory exchange between passes; the pass-2/3
 //     twiddles of a thread stay in registers for the whole kernel.
-//   * BK_i's 48 KB (own rows x outputs o, o2) are TMA-staged two steps ahead; partials and halves move CTA-to-CTA with
-//     shared::cluster bulk copies that complete on the receiver's mbarrier (double-buffered by step parity,
-//     safe for the same reason as br9's hand-over: a CTA can only send for step i+2 after it has received the
-//     receiver's data of step i+1, which the receiver produced after consuming step i).
+//   * BK_i's 48 KB (own rows x outputs o, o2) are TMA-staged two steps ahead.
 #include "tb_fft.cuh"
 #include "tb_kernels.cuh"
 
@@ -29,7 +31,6 @@ constexpr int kLMacIt = (512 + kLThreads - 1) / kLThreads;
 #define TB_BRL_BK_ISSUER 64
 #endif
 constexpr int kBkIssuer = TB_BRL_BK_ISSUER;   // thread that issues the per-step BK TMA (outside warps 0-1)
-constexpr int kPsumPusher = 224;                // thread (warp 7) that pushes the partial
 constexpr uint32_t kRowsBytes = 512 * 16;   // the partner's partial MAC of this CTA's output (512 complex)
 
 #ifdef TB_BRL_TRACE   // scratch instrumentation (tools/buildvar.sh WORK name -DTB_BRL_TRACE): clock64 per phase
@@ -43,7 +44,6 @@ __device__ long long g_brl_trace[4][8][16];
 struct __align__(128) BrlSmem {
     double2 bk[2][kRows][512];                 // BK_i, rows 0..5 of output o = 2q + h, by step parity (96 KB)
     double2 dslot[kL][512];                    // own forward rows (bloc q), swizzled positions
-    double2 psend[512];                        // partial MAC of the partner's output over the own rows
     double2 precv[2][512];                     // the partner's partial MAC of this CTA's output, by step parity
     double2 oslot[512];                        // MAC output, then the inverse's exchange buffer
     uint32_t res[kN];                          // own rounded half of the product (sent to the sibling)
@@ -304,13 +304,14 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
                     s2.re = fma(d.re, b2.re, fma(-d.im, b2.im, s2.re));
                     s2.im = fma(d.re, b2.im, fma(d.im, b2.re, s2.im));
                 }
-                stc(&S.psend[k], s2);
+                // straight from registers into the partner's precv[buf], completing on its mbarrier
+                asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f64 [%0], {%1, %2}, [%3];" ::"r"(
+                                 rows_dst + (uint32_t)((buf * 512 + k) * 16)),
+                             "d"(s2.re), "d"(s2.im), "r"(rows_mb + (uint32_t)(buf * 8))
+                             : "memory");
             }
             m3[e] = s;
         }
-        __syncthreads();                                  // psend complete
-        if (tid == kPsumPusher)
-            push_peer(rows_dst + (uint32_t)(buf * 512 * 16), S.psend, 512 * 16, rows_mb + (uint32_t)(buf * 8));
         mb_wait(&S.mbar_rows[buf], par);
         BRL_T(3)
 #pragma unroll
@@ -321,7 +322,6 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
                 stc(&S.oslot[lsw(k)], dcplx{m3[e].re + pr.re, m3[e].im + pr.im});
             }
         }
-        if (tid == kPsumPusher) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // psend read
         __syncthreads();                                  // bk[buf], precv[buf] consumed; oslot complete
         BRL_T(4)
         // step i + 2's BK and the expectation of its rows: issued by a thread of warp 2, idle during the inverse
@@ -339,11 +339,19 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
 #pragma unroll
             for (int v = 0; v < 8; v++) {
                 const int c = gp1(tt, v);
-                S.res[c] = round_mod32(x[v].re) << (16 * h);
-                S.res[c + 512] = round_mod32(x[v].im) << (16 * h);
+                const uint32_t lo = round_mod32(x[v].re) << (16 * h), hi = round_mod32(x[v].im) << (16 * h);
+                S.res[c] = lo;
+                S.res[c + 512] = hi;
+                // and straight into the sibling's rres[buf] (4 KB per step, completing on its mbarrier)
+                asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b32 [%0], %1, [%2];" ::"r"(
+                                 res_dst + (uint32_t)((buf * kN + c) * 4)),
+                             "r"(lo), "r"(res_mb + (uint32_t)(buf * 8))
+                             : "memory");
+                asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b32 [%0], %1, [%2];" ::"r"(
+                                 res_dst + (uint32_t)((buf * kN + c + 512) * 4)),
+                             "r"(hi), "r"(res_mb + (uint32_t)(buf * 8))
+                             : "memory");
             }
-            bar_pair(4);
-            if (tid == 0) push_peer(res_dst + (uint32_t)(buf * kN * 4), S.res, kN * 4, res_mb + (uint32_t)(buf * 8));
         }
         __syncthreads();
         BRL_T(5)
@@ -359,7 +367,6 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         BRL_T(7)
         if (tid == 0) {   // (no barrier after this: warps 0-1 rewrite res only after the next phase-A barrier,
                           // which tid 0 reaches after the wait; the expect precedes tid 0's own next push)
-            asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // res readable again
             if (i + 2 < kn) mb_expect(&S.mbar_res[buf], kN * 4);            // the sibling's half of step i + 2
         }
     }
