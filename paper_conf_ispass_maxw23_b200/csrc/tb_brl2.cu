@@ -3,8 +3,10 @@
 //
 // brl's arithmetic, transforms and hand-over protocol (tb_brl.cu, same exact FFT-domain products, bit-identical
 // output) with the cluster halved: CTA q (rank q) owns output polynomial q and BOTH 16-bit BK halves h, so
-//   * it computes the 3 digit rows of ACC[q] (3 forward transforms on warp pairs 0-2) and pushes them to CTA 1-q,
-//   * its MAC produces both outputs o = 2q + h (each digit row read once for the two halves),
+//   * it computes the 3 digit rows of ACC[q] (3 forward transforms on warp pairs 0-2),
+//   * its MAC is split by bloc like brl's: the own rows times BK_i for the partner's two outputs 2(1-q) + h go to
+//     CTA 1-q per thread with st.async (16 KB; round 1 pushed the three rows, 24 KB, with bulk copies), then the
+//     own rows for the own outputs o = 2q + h, plus the partner's partials of those (1.92 -> 1.82 ms for one gate),
 //   * warp pairs 0 and 1 run the two inverse transforms side by side (h = 0, 1), and the halves meet locally:
 //     ACC[q] += lo + 2^16 hi with no second hand-over.
 // Per CMux step that is brl's forward phase, twice its MAC, the same inverse latency (two transforms in parallel
@@ -20,7 +22,7 @@ namespace tb {
 struct __align__(128) Brl2Smem {
     double2 bk[2][kRows][512];                 // BK_i rows 0..5 of outputs o = 2q + h, h = 0, 1 (96 KB)
     double2 dslot[kL][512];                    // own forward rows (bloc q), swizzled positions
-    double2 rrows[2][kL][512];                 // rows of bloc 1-q from CTA 1-q, by step parity
+    double2 precv[2][2][512];                  // the partner's partial MACs of this CTA's outputs, by step parity
     double2 oslot[2][512];                     // MAC outputs (h = 0, 1), then the inverses' exchange buffers
     uint32_t res[2][kN];                       // rounded halves, h = 0 (lo) and 1 (hi, << 16)
     uint32_t acc[3 * kN];                      // ACC[q] as (acc, -acc, acc)
@@ -28,19 +30,22 @@ struct __align__(128) Brl2Smem {
     unsigned long long mbar_bk, mbar_rows[2];
 };
 
-// BK_i rows 0..5 of outputs 2q, 2q + 1 -> bk (one thread)
+// BK_i -> bk (one thread): slot (h, r) = the own bloc's row 3q + (r mod 3) of output 2q + h (r < 3) and of the
+// partner's output 2(1-q) + h (r >= 3)
 __device__ __forceinline__ void issue_bk_l2(Brl2Smem& S, const double2* bkf, int i, int q) {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     mb_expect(&S.mbar_bk, 2 * kRows * 512 * 16);
 #pragma unroll
     for (int h = 0; h < 2; h++)
 #pragma unroll
-        for (int r = 0; r < kRows; r++)
+        for (int r = 0; r < kRows; r++) {
+            const size_t row = (size_t)(i * kRows + kL * q + r % kL) * 4 + (r < kL ? 2 * q + h : 2 * (1 - q) + h);
             asm volatile(
                 "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                     sm32(S.bk[h][r])),
-                "l"(bkf + ((size_t)(i * kRows + r) * 4 + 2 * q + h) * 512), "r"(512 * 16), "r"(sm32(&S.mbar_bk))
+                "l"(bkf + row * 512), "r"(512 * 16), "r"(sm32(&S.mbar_bk))
                 : "memory");
+        }
 }
 
 constexpr int kBk2Issuer = 128;   // issues the per-step BK TMA: warp 4 has no inverse to run
@@ -58,7 +63,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
         mb_init(&S.mbar_bk);
         for (int b = 0; b < 2; b++) mb_init(&S.mbar_rows[b]);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        for (int b = 0; b < 2; b++) mb_expect(&S.mbar_rows[b], kL * 512 * 16);   // rows of steps 0 and 1
+        for (int b = 0; b < 2; b++) mb_expect(&S.mbar_rows[b], 2 * 512 * 16);   // partials of steps 0 and 1
     }
     __syncthreads();
     if (tid == 0) issue_bk_l2(S, bkf, 0, q);
@@ -100,7 +105,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
     t3.a = ldc(twL + tt * 6 + 3);
     t3.b = ldc(twL + tt * 6 + 4);
     t3.c = ldc(twL + tt * 6 + 5);
-    const uint32_t rows_dst = cl_map(sm32(&S.rrows[0][0][0]), rank ^ 1u);
+    const uint32_t rows_dst = cl_map(sm32(&S.precv[0][0][0]), rank ^ 1u);
     const uint32_t rows_mb = cl_map(sm32(&S.mbar_rows[0]), rank ^ 1u);
 
     for (int i = 0; i < kn; i++) {
@@ -118,24 +123,38 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
                 x[v] = dcplx{small_to_double((u0 >> shift) & 127u, 64.0), small_to_double((u1 >> shift) & 127u, 64.0)};
             }
             fwd2w(x, S.dslot[jd], t1, t2, t3, tt, 1 + jd);
-            bar_pair(1 + jd);
-            if (tt == 0)   // row jd -> CTA 1-q as soon as this warp pair is done
-                push_peer(rows_dst + (uint32_t)((buf * kL + jd) * 512 * 16), &S.dslot[jd][0], 512 * 16,
-                          rows_mb + (uint32_t)(buf * 8));
         }
         __syncthreads();
         mb_wait(&S.mbar_bk, (uint32_t)(i & 1));
-        // ---- B: out_h[k] = sum_{r<6} D_r[k] BK_i[r][2q + h][k]; own bloc's rows first, then the other bloc's ----
+        // ---- B: the MAC split by bloc (brl's partial exchange): own rows x BK_i for the own outputs 2q + h and for
+        // the partner's outputs 2(1-q) + h; the partner's partials go out per thread with st.async (16 KB) ----
         dcplx m3[kLMacIt][2];
 #pragma unroll
         for (int e = 0; e < kLMacIt; e++) {
             const int k = tid + kLThreads * e;
-            dcplx s0 = {0.0, 0.0}, s1 = {0.0, 0.0};
+            dcplx s0 = {0.0, 0.0}, s1 = {0.0, 0.0}, p0 = {0.0, 0.0}, p1 = {0.0, 0.0};
             if (k < 512) {
 #pragma unroll
                 for (int r = 0; r < kL; r++) {
                     const dcplx d = ldc(&S.dslot[r][lsw(k)]);
-                    const dcplx b0 = ldc(&S.bk[0][q * kL + r][k]), b1 = ldc(&S.bk[1][q * kL + r][k]);
+                    const dcplx c0 = ldc(&S.bk[0][kL + r][k]), c1 = ldc(&S.bk[1][kL + r][k]);
+                    p0.re = fma(d.re, c0.re, fma(-d.im, c0.im, p0.re));
+                    p0.im = fma(d.re, c0.im, fma(d.im, c0.re, p0.im));
+                    p1.re = fma(d.re, c1.re, fma(-d.im, c1.im, p1.re));
+                    p1.im = fma(d.re, c1.im, fma(d.im, c1.re, p1.im));
+                }
+                asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f64 [%0], {%1, %2}, [%3];" ::"r"(
+                                 rows_dst + (uint32_t)(((buf * 2 + 0) * 512 + k) * 16)),
+                             "d"(p0.re), "d"(p0.im), "r"(rows_mb + (uint32_t)(buf * 8))
+                             : "memory");
+                asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f64 [%0], {%1, %2}, [%3];" ::"r"(
+                                 rows_dst + (uint32_t)(((buf * 2 + 1) * 512 + k) * 16)),
+                             "d"(p1.re), "d"(p1.im), "r"(rows_mb + (uint32_t)(buf * 8))
+                             : "memory");
+#pragma unroll
+                for (int r = 0; r < kL; r++) {
+                    const dcplx d = ldc(&S.dslot[r][lsw(k)]);
+                    const dcplx b0 = ldc(&S.bk[0][r][k]), b1 = ldc(&S.bk[1][r][k]);
                     s0.re = fma(d.re, b0.re, fma(-d.im, b0.im, s0.re));
                     s0.im = fma(d.re, b0.im, fma(d.im, b0.re, s0.im));
                     s1.re = fma(d.re, b1.re, fma(-d.im, b1.im, s1.re));
@@ -150,24 +169,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
         for (int e = 0; e < kLMacIt; e++) {
             const int k = tid + kLThreads * e;
             if (k < 512) {
-                dcplx s0 = m3[e][0], s1 = m3[e][1];
-#pragma unroll
-                for (int r = 0; r < kL; r++) {
-                    const dcplx d = ldc(&S.rrows[buf][r][lsw(k)]);
-                    const dcplx b0 = ldc(&S.bk[0][(1 - q) * kL + r][k]), b1 = ldc(&S.bk[1][(1 - q) * kL + r][k]);
-                    s0.re = fma(d.re, b0.re, fma(-d.im, b0.im, s0.re));
-                    s0.im = fma(d.re, b0.im, fma(d.im, b0.re, s0.im));
-                    s1.re = fma(d.re, b1.re, fma(-d.im, b1.im, s1.re));
-                    s1.im = fma(d.re, b1.im, fma(d.im, b1.re, s1.im));
-                }
-                stc(&S.oslot[0][lsw(k)], s0);
-                stc(&S.oslot[1][lsw(k)], s1);
+                const dcplx r0 = ldc(&S.precv[buf][0][k]), r1 = ldc(&S.precv[buf][1][k]);
+                stc(&S.oslot[0][lsw(k)], dcplx{m3[e][0].re + r0.re, m3[e][0].im + r0.im});
+                stc(&S.oslot[1][lsw(k)], dcplx{m3[e][1].re + r1.re, m3[e][1].im + r1.im});
             }
         }
-        if ((tid & 63) == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // dslot rows sent
         __syncthreads();                                  // bk, rrows[buf] consumed; oslot complete
         if (tid == kBk2Issuer) {   // a thread of warp 4, idle during the two inverses (warp pairs 0 and 1)
-            if (i + 2 < kn) mb_expect(&S.mbar_rows[buf], kL * 512 * 16);   // rows of step i + 2
+            if (i + 2 < kn) mb_expect(&S.mbar_rows[buf], 2 * 512 * 16);    // partials of step i + 2
             if (i + 1 < kn) issue_bk_l2(S, bkf, i + 1, q);                  // lands during C and the next A
         }
         if (jd < 2) {   // ---- C: inverse of half h = jd (warp pair jd), round, << 16 h ----
