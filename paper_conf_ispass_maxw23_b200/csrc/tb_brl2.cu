@@ -174,7 +174,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
                 stc(&S.oslot[1][lsw(k)], dcplx{m3[e][1].re + r1.re, m3[e][1].im + r1.im});
             }
         }
-        __syncthreads();                                  // bk, rrows[buf] consumed; oslot complete
+        __syncthreads();                                  // bk, precv[buf] consumed; oslot complete
         if (tid == kBk2Issuer) {   // a thread of warp 4, idle during the two inverses (warp pairs 0 and 1)
             if (i + 2 < kn) mb_expect(&S.mbar_rows[buf], 2 * 512 * 16);    // partials of step i + 2
             if (i + 1 < kn) issue_bk_l2(S, bkf, i + 1, q);                  // lands during C and the next A
