@@ -6,20 +6,23 @@
 // shorten the serial chain of 630 steps that bounds a narrow netlist level:
 //   * CTA (q, h) of the cluster (rank 2q + h) owns output polynomial q and BK half h: it computes the 3 digit
 //     rows of ACC[q] (the two CTAs of a q compute them redundantly) and splits the MAC by bloc (it is linear):
-//     its own rows times BK_i for its output o = 2q + h and for the partner CTA (1-q, h)'s output o2; it sends
-//     the o2 partial (8 KB; round 1 sent the three rows, 24 KB, and multiplied the received rows itself), adds
-//     the partner's partial of o, and runs one inverse transform; the two CTAs of a q swap their rounded halves
+//     its own rows times BK_i for its output o = 2q + h and, for half of the positions ([256 h, 256 h + 256)),
+//     for both outputs of the other bloc; it sends each of those two partials (4 KB) to the CTA that owns the
+//     output, receives its own output's other-bloc partial from both CTAs of bloc 1-q (8 KB; round 1 sent the
+//     three rows, 24 KB, and multiplied the received rows itself), and runs one inverse transform; the two CTAs
+//     of a q swap their rounded halves
 //     and both add lo + 2^16 hi into their copy of ACC[q].  The summation order differs from the other
 //     variants; the FP64 error bound does not depend on it, so the rounded products are identical.
 //   * both hand-overs are per-thread st.async stores straight from registers into the peer's shared memory,
 //     completing on its mbarrier (no staging buffer, no barrier and proxy fence before a bulk copy: one-gate
-//     level 1.79 -> 1.64 ms), double-buffered by step parity (safe for the same reason as br9's
-//     hand-over: a CTA can only send for step i+2 after it has received the receiver's data of step i+1, which
-//     the receiver produced after consuming step i).
+//     level 1.79 -> 1.58 ms), double-buffered by step parity (safe for the same reason as br9's
+//     hand-over: a CTA can only send for step i+2 after it has received the receiver's data of step i+1 -- both
+//     CTAs of the other bloc send to both of this bloc -- which the receiver produced after consuming step i).
 //   * every transform is split over 2 warps (64 threads x 8 values) and done as three radix-8 passes (stages
 //     1-3, 4-6, 7-9 of the merged-twist tree), with one shared-memory exchange between passes; the pass-2/3
 //     twiddles of a thread stay in registers for the whole kernel.
-//   * BK_i's 48 KB (own rows x outputs o, o2) are TMA-staged two steps ahead.
+//   * BK_i's 48 KB (own rows x output o, and x the other bloc's outputs on half the positions) are TMA-staged
+//     two steps ahead.
 #include "tb_fft.cuh"
 #include "tb_kernels.cuh"
 
@@ -31,7 +34,7 @@ constexpr int kLMacIt = (512 + kLThreads - 1) / kLThreads;
 #define TB_BRL_BK_ISSUER 64
 #endif
 constexpr int kBkIssuer = TB_BRL_BK_ISSUER;   // thread that issues the per-step BK TMA (outside warps 0-1)
-constexpr uint32_t kRowsBytes = 512 * 16;   // the partner's partial MAC of this CTA's output (512 complex)
+constexpr uint32_t kRowsBytes = 512 * 16;   // the other bloc's partial MAC of this CTA's output (512 complex)
 
 #ifdef TB_BRL_TRACE   // scratch instrumentation (tools/buildvar.sh WORK name -DTB_BRL_TRACE): clock64 per phase
 __device__ long long g_brl_trace[4][8][16];
@@ -178,14 +181,27 @@ __device__ __forceinline__ void push_peer(uint32_t dst, const void* src, uint32_
         : "memory");
     asm volatile("cp.async.bulk.commit_group;" ::: "memory");
 }
-// BK_i -> bk[buf] (one thread): the own bloc's rows 3q..3q+2 of output o (slots 0-2) and of the partner's output
-// o2 (slots 3-5).
-__device__ __forceinline__ void issue_bk_l(BrlSmem& S, const double2* bkf, int i, int o, int o2, int q, int buf) {
+// BK_i -> bk[buf] (one thread): the own bloc's rows 3q..3q+2 of output o (slots 0-2) and, for positions
+// [256 h, 256 h + 256), of the other bloc's two outputs 2(1-q) + 0 and + 1 (slots 3-5, one half each).
+__device__ __forceinline__ void issue_bk_l(BrlSmem& S, const double2* bkf, int i, int o, int q, int h,
+                                           int buf) {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     mb_expect(&S.mbar_bk[buf], kRows * 512 * 16);
 #pragma unroll
     for (int r = 0; r < kRows; r++) {
-        const size_t row = (size_t)(i * kRows + kL * q + r % kL) * 4 + (r < kL ? o : o2);
+        if (r >= kL) {
+            // slot r: the partner bloc's outputs 2(1-q) + 0 and + 1, positions [256 h, 256 h + 256) of each
+#pragma unroll
+            for (int hh = 0; hh < 2; hh++)
+                asm volatile(
+                    "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                        sm32(&S.bk[buf][r][256 * hh])),
+                    "l"(bkf + ((size_t)(i * kRows + kL * q + r % kL) * 4 + 2 * (1 - q) + hh) * 512 + 256 * h),
+                    "r"(256 * 16), "r"(sm32(&S.mbar_bk[buf]))
+                    : "memory");
+            continue;
+        }
+        const size_t row = (size_t)(i * kRows + kL * q + r) * 4 + o;
         asm volatile(
             "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                 sm32(S.bk[buf][r])),
@@ -203,7 +219,6 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint32_t rank = cl_rank();
     const int q = (int)(rank >> 1), h = (int)(rank & 1), o = 2 * q + h;
-    const int o2 = 2 * (1 - q) + h;                      // output of the partner CTA (1-q, h)
     const int gl = blockIdx.x >> 2;                      // one lane (bootstrap) per cluster
 
     if (tid == 0) {
@@ -220,8 +235,8 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
     }
     __syncthreads();
     if (tid == 0) {
-        issue_bk_l(S, bkf, 0, o, o2, q, 0);
-        issue_bk_l(S, bkf, 1, o, o2, q, 1);
+        issue_bk_l(S, bkf, 0, o, q, h, 0);
+        issue_bk_l(S, bkf, 1, o, q, h, 1);
     }
     {   // a1, a2 (every CTA of the cluster)
         LaneDesc d = {0, -1, 0, 0, 0u, 0u, 0u, 0u};
@@ -262,6 +277,8 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
     t3.c = ldc(twL + tt * 6 + 5);
     const uint32_t rows_dst = cl_map(sm32(&S.precv[0][0]), rank ^ 2u);
     const uint32_t rows_mb = cl_map(sm32(&S.mbar_rows[0]), rank ^ 2u);
+    const uint32_t rows_dst_x = cl_map(sm32(&S.precv[0][0]), rank ^ 3u);   // CTA (1-q, 1-h)
+    const uint32_t rows_mb_x = cl_map(sm32(&S.mbar_rows[0]), rank ^ 3u);
     const uint32_t res_dst = cl_map(sm32(&S.rres[0][0]), rank ^ 1u);
     const uint32_t res_mb = cl_map(sm32(&S.mbar_res[0]), rank ^ 1u);
 
@@ -287,28 +304,49 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         mb_wait(&S.mbar_bk[buf], par);
         BRL_T(2)
         // ---- B: the MAC split by bloc (it is linear): this CTA multiplies its own rows (bloc q) by BK_i for its
-        // output o and for the partner's output o2, sends the o2 partial (8 KB instead of 24 KB of rows), and adds
-        // the partner's partial of o.  Round-off: the FP64 error bound of §5b holds for any summation order. ----
+        // output o on all positions and for the other bloc's two outputs on positions [256 h, 256 h + 256), sends
+        // those two partials (4 KB each) to their owners, and adds the other bloc's partial of o, received half
+        // from each CTA of bloc 1-q.  Round-off: the FP64 error bound of 5b holds for any summation order. ----
+        // the partners' partials first: positions [256 h, 256 h + 256) of both outputs of bloc 1-q, one to each of
+        // CTA (1-q, h) and (1-q, 1-h); each receives its 8 KB half from two senders at once
+        dcplx dr[kLMacIt][kL];
+#pragma unroll
+        for (int e = 0; e < kLMacIt; e++) {
+            const int k = tid + kLThreads * e;
+#pragma unroll
+            for (int r = 0; r < kL; r++) dr[e][r] = ldc(&S.dslot[r][lsw(k)]);
+        }
+        {
+            const int k = tid + kLThreads * h;
+            const dcplx d0 = h ? dr[1][0] : dr[0][0], d1 = h ? dr[1][1] : dr[0][1], d2 = h ? dr[1][2] : dr[0][2];
+#pragma unroll
+            for (int hh = 0; hh < 2; hh++) {
+                dcplx s2 = {0.0, 0.0};
+#pragma unroll
+                for (int r = 0; r < kL; r++) {
+                    const dcplx d = r == 0 ? d0 : (r == 1 ? d1 : d2), b2 = ldc(&S.bk[buf][kL + r][256 * hh + tid]);
+                    s2.re = fma(d.re, b2.re, fma(-d.im, b2.im, s2.re));
+                    s2.im = fma(d.re, b2.im, fma(d.im, b2.re, s2.im));
+                }
+                const bool same = hh == h;
+                asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f64 [%0], {%1, %2}, [%3];" ::"r"(
+                                 (same ? rows_dst : rows_dst_x) + (uint32_t)((buf * 512 + k) * 16)),
+                             "d"(s2.re), "d"(s2.im), "r"((same ? rows_mb : rows_mb_x) + (uint32_t)(buf * 8))
+                             : "memory");
+            }
+        }
         dcplx m3[kLMacIt];
 #pragma unroll
         for (int e = 0; e < kLMacIt; e++) {
             const int k = tid + kLThreads * e;
-            dcplx s = {0.0, 0.0}, s2 = {0.0, 0.0};
+            dcplx s = {0.0, 0.0};
             if (k < 512) {
 #pragma unroll
                 for (int r = 0; r < kL; r++) {
-                    const dcplx d = ldc(&S.dslot[r][lsw(k)]);
-                    const dcplx b = ldc(&S.bk[buf][r][k]), b2 = ldc(&S.bk[buf][kL + r][k]);
+                    const dcplx d = dr[e][r], b = ldc(&S.bk[buf][r][k]);
                     s.re = fma(d.re, b.re, fma(-d.im, b.im, s.re));
                     s.im = fma(d.re, b.im, fma(d.im, b.re, s.im));
-                    s2.re = fma(d.re, b2.re, fma(-d.im, b2.im, s2.re));
-                    s2.im = fma(d.re, b2.im, fma(d.im, b2.re, s2.im));
                 }
-                // straight from registers into the partner's precv[buf], completing on its mbarrier
-                asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f64 [%0], {%1, %2}, [%3];" ::"r"(
-                                 rows_dst + (uint32_t)((buf * 512 + k) * 16)),
-                             "d"(s2.re), "d"(s2.im), "r"(rows_mb + (uint32_t)(buf * 8))
-                             : "memory");
             }
             m3[e] = s;
         }
@@ -330,7 +368,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         if (tid == kBkIssuer) {
             if (i + 2 < kn) {
                 mb_expect(&S.mbar_rows[buf], kRowsBytes);                     // rows / partial of step i + 2
-                issue_bk_l(S, bkf, i + 2, o, o2, q, buf);
+                issue_bk_l(S, bkf, i + 2, o, q, h, buf);
             }
         }
         if (warp < 2) {   // ---- C: inverse (warp pair 0), round, << 16 h ----
