@@ -1,7 +1,7 @@
 #!/bin/bash
 # Round-2 session-2 final batch (one B200): full GPU suite, smoke, latency table, bench line, reference arm,
-# BR DRAM traffic at the bench size, launch list of the default command, every BASELINE config, sanitizers
-# (memcheck / synccheck over the full set, racecheck on the latency kernels whose step loop changed).
+# BR DRAM traffic at the bench size, launch list of the default command, every BASELINE config.
+# (compute-sanitizer is closed on this GPU pool since round 2 session 2: not run.)
 O=gpurun_out
 T=${TAG:-r02s2}
 timeout 1800 python -m pytest tests -m gpu -q > $O/${T}_gpu_tests.log 2>&1; echo "exit $?" >> $O/${T}_gpu_tests.log
@@ -15,8 +15,4 @@ timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_d
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/${T}_launches.csv \
     python bench.py --no-cpu-baseline --steps 2 --warmup 3 > /dev/null 2>&1
 timeout 1500 python tools/workloads.py > $O/${T}_workloads.jsonl 2> $O/${T}_workloads.err
-for tool in memcheck synccheck; do
-  TB_SAN_NOBRT=$([ $tool = synccheck ] && echo 1 || echo 0) timeout 1500 compute-sanitizer --tool $tool python tools/sanitize_run.py > $O/${T}_sanitize_$tool.log 2>&1
-done
-TB_SAN_LATENCY=1 timeout 1200 compute-sanitizer --tool racecheck python tools/sanitize_run.py > $O/${T}_sanitize_racecheck_lat.log 2>&1
 echo done
