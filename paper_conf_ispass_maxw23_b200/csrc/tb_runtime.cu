@@ -13,8 +13,18 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>   // header-only NVTX v3: ranges cost a branch unless a tool (nsys, ncu) is attached
 #include "../../include/tfhe_b200.h"
 #include "tb_kernels.cuh"
+
+namespace {
+// NVTX range over one C-ABI call (levels, gate batches, host-buffer netlists), so that a profiler timeline groups
+// each call's kernels
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
+}  // namespace
 
 
 using namespace tb;
@@ -575,6 +585,7 @@ static int run_ks(tb_ctx* c, const uint32_t* lanes, int64_t lane_base, int64_t l
 
 extern "C" int tb_gates(tb_ctx* c, int gate, const uint32_t* ca, const uint32_t* cb, const uint32_t* cc,
                         uint32_t* out, int64_t count, int64_t stride, tb_stream stream) {
+    NvtxRange nv("tb_gates");
     int rc = check_ready(c);
     if (rc) return rc;
     if (count < 0 || stride < kn + 1 || count > ((int64_t)1 << 29)) return fail(TB_EINVAL, "bad count or stride");
@@ -1108,6 +1119,7 @@ extern "C" int tb_netlist_level(const tb_dev_netlist* d, int64_t level, int64_t*
 
 extern "C" int tb_run_level(tb_ctx* c, const tb_dev_netlist* d, int64_t level, int64_t g0, int64_t g1,
                             uint32_t* wires, int64_t stride, tb_stream stream) {
+    NvtxRange nv("tb_run_level");
     int rc = check_ready(c);
     if (rc) return rc;
     if (!d || !wires) return fail(TB_EINVAL, "null argument");
@@ -1259,6 +1271,7 @@ static int run_netlist_host_impl(tb_ctx* c, const tb_dev_netlist* d, const uint3
 constexpr int64_t kHostChunkMinWaves = 8, kHostEdgeWaves = 3;
 extern "C" int tb_run_netlist_host(tb_ctx* c, const tb_dev_netlist* d, const uint32_t* hin, int64_t in_stride,
                                    const int64_t* outw, int64_t n_out, uint32_t* hout, int64_t out_stride) {
+    NvtxRange nv("tb_run_netlist_host");
     const int rc = run_netlist_host_impl(c, d, hin, in_stride, outw, n_out, hout, out_stride);
     if (rc != TB_OK && c) {   // no copy from / into the caller's host buffers may still be in flight on return
         for (cudaStream_t s : {c->own, c->h2d, c->d2h})
