@@ -54,6 +54,30 @@ __global__ void __launch_bounds__(512, 1) kern(double* sink, const double2* gsrc
                 asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(smem_u32(p)), "d"(a[i]), "d"(a[(i + 1) & 15]) : "memory");
             }
             a[it & 15] += 1.0;
+        } else if (MODE == 10) {   // STS.64: 32 per iteration (same bytes as 16 STS.128)
+#pragma unroll
+            for (int i = 0; i < 16; i++) {
+                double* p = reinterpret_cast<double*>(&buf[((it + warp * 16 + i) & 63) * 32 + lane]);
+                asm volatile("st.shared.f64 [%0], %1;" ::"r"(smem_u32(p)), "d"(a[i]) : "memory");
+                asm volatile("st.shared.f64 [%0], %1;" ::"r"(smem_u32(p + 1)), "d"(a[(i + 1) & 15]) : "memory");
+            }
+            a[it & 15] += 1.0;
+        } else if (MODE == 11) {   // STS.32: 64 per iteration (same bytes)
+#pragma unroll
+            for (int i = 0; i < 16; i++) {
+                float* p = reinterpret_cast<float*>(&buf[((it + warp * 16 + i) & 63) * 32 + lane]);
+#pragma unroll
+                for (int w = 0; w < 4; w++)
+                    asm volatile("st.shared.b32 [%0], %1;" ::"r"(smem_u32(p + w)), "r"(__double2loint(a[(i + w) & 15])) : "memory");
+            }
+            a[it & 15] += 1.0;
+        } else if (MODE == 12) {   // STS.128 with a 16-B lane stride but lanes permuted within 8-lane groups
+#pragma unroll
+            for (int i = 0; i < 16; i++) {
+                double2* p = &buf[((it + warp * 16 + i) & 63) * 32 + (lane ^ (i & 7))];
+                asm volatile("st.shared.v2.f64 [%0], {%1, %2};" ::"r"(smem_u32(p)), "d"(a[i]), "d"(a[(i + 1) & 15]) : "memory");
+            }
+            a[it & 15] += 1.0;
         } else if (MODE == 4) {   // LDG.128 from a 32 KB block (L1 resident): 16 per iteration
 #pragma unroll
             for (int i = 0; i < 16; i++) {
@@ -172,5 +196,9 @@ int main() {
     run<7>("mix_DFMA64_LDS128x16 (DFMA count)", 64, sink, g, cyc, nsm);
     run<8>("mix_DFMA64_SHFLx32 (DFMA count)", 64, sink, g, cyc, nsm);
     run<9>("mix_DFMA64_LDG128x16 (DFMA count)", 64, sink, g, cyc, nsm);
+    run<10>("STS.64 (x2 per 16 B)", 32, sink, g, cyc, nsm);
+    run<11>("STS.32 (x4 per 16 B)", 64, sink, g, cyc, nsm);
+    run<12>("STS.128 lane-permuted", 16, sink, g, cyc, nsm);
+    run<3>("STS.128 (again)", 16, sink, g, cyc, nsm);
     return 0;
 }
