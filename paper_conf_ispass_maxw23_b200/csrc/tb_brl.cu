@@ -34,7 +34,7 @@ constexpr int kLMacIt = (512 + kLThreads - 1) / kLThreads;
 #define TB_BRL_BK_ISSUER 64
 #endif
 constexpr int kBkIssuer = TB_BRL_BK_ISSUER;   // thread that issues the per-step BK TMA (outside warps 0-1)
-constexpr uint32_t kRowsBytes = 512 * 16;   // the other bloc's partial MAC of this CTA's output (512 complex)
+constexpr uint32_t kPartBytes = 512 * 16;   // the other bloc's partial MAC of this CTA's output (512 complex)
 
 #ifdef TB_BRL_TRACE   // scratch instrumentation (tools/buildvar.sh WORK name -DTB_BRL_TRACE): clock64 per phase
 __device__ long long g_brl_trace[4][8][16];
@@ -45,7 +45,7 @@ __device__ long long g_brl_trace[4][8][16];
 #endif
 
 struct __align__(128) BrlSmem {
-    double2 bk[2][kRows][512];                 // BK_i, rows 0..5 of output o = 2q + h, by step parity (96 KB)
+    double2 bk[2][kRows][512];                 // BK_i (issue_bk_l), by step parity (96 KB)
     double2 dslot[kL][512];                    // own forward rows (bloc q), swizzled positions
     double2 precv[2][512];                     // the partner's partial MAC of this CTA's output, by step parity
     double2 oslot[512];                        // MAC output, then the inverse's exchange buffer
@@ -53,7 +53,7 @@ struct __align__(128) BrlSmem {
     uint32_t rres[2][kN];                      // the sibling's half, by step parity
     uint32_t acc[3 * kN];                      // ACC[q] as (acc, -acc, acc)
     uint16_t bar[kn + 2];
-    unsigned long long mbar_bk[2], mbar_rows[2], mbar_res[2];
+    unsigned long long mbar_bk[2], mbar_part[2], mbar_res[2];
 };
 
 // swizzled slot of transform position k: each of the three pass groupings below touches 8 distinct 16-byte
@@ -224,12 +224,12 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
     if (tid == 0) {
         for (int b = 0; b < 2; b++) {
             mb_init(&S.mbar_bk[b]);
-            mb_init(&S.mbar_rows[b]);
+            mb_init(&S.mbar_part[b]);
             mb_init(&S.mbar_res[b]);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        for (int b = 0; b < 2; b++) {                    // rows and halves of steps 0 and 1 may arrive any time
-            mb_expect(&S.mbar_rows[b], kRowsBytes);
+        for (int b = 0; b < 2; b++) {                    // partials and halves of steps 0 and 1 may arrive any time
+            mb_expect(&S.mbar_part[b], kPartBytes);
             mb_expect(&S.mbar_res[b], kN * 4);
         }
     }
@@ -275,10 +275,10 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
     t3.a = ldc(twL + tt * 6 + 3);
     t3.b = ldc(twL + tt * 6 + 4);
     t3.c = ldc(twL + tt * 6 + 5);
-    const uint32_t rows_dst = cl_map(sm32(&S.precv[0][0]), rank ^ 2u);
-    const uint32_t rows_mb = cl_map(sm32(&S.mbar_rows[0]), rank ^ 2u);
-    const uint32_t rows_dst_x = cl_map(sm32(&S.precv[0][0]), rank ^ 3u);   // CTA (1-q, 1-h)
-    const uint32_t rows_mb_x = cl_map(sm32(&S.mbar_rows[0]), rank ^ 3u);
+    const uint32_t part_dst = cl_map(sm32(&S.precv[0][0]), rank ^ 2u);
+    const uint32_t part_mb = cl_map(sm32(&S.mbar_part[0]), rank ^ 2u);
+    const uint32_t part_dst_x = cl_map(sm32(&S.precv[0][0]), rank ^ 3u);   // CTA (1-q, 1-h)
+    const uint32_t part_mb_x = cl_map(sm32(&S.mbar_part[0]), rank ^ 3u);
     const uint32_t res_dst = cl_map(sm32(&S.rres[0][0]), rank ^ 1u);
     const uint32_t res_mb = cl_map(sm32(&S.mbar_res[0]), rank ^ 1u);
 
@@ -330,8 +330,8 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
                 }
                 const bool same = hh == h;
                 asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f64 [%0], {%1, %2}, [%3];" ::"r"(
-                                 (same ? rows_dst : rows_dst_x) + (uint32_t)((buf * 512 + k) * 16)),
-                             "d"(s2.re), "d"(s2.im), "r"((same ? rows_mb : rows_mb_x) + (uint32_t)(buf * 8))
+                                 (same ? part_dst : part_dst_x) + (uint32_t)((buf * 512 + k) * 16)),
+                             "d"(s2.re), "d"(s2.im), "r"((same ? part_mb : part_mb_x) + (uint32_t)(buf * 8))
                              : "memory");
             }
         }
@@ -350,7 +350,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
             }
             m3[e] = s;
         }
-        mb_wait(&S.mbar_rows[buf], par);
+        mb_wait(&S.mbar_part[buf], par);
         BRL_T(3)
 #pragma unroll
         for (int e = 0; e < kLMacIt; e++) {
@@ -367,7 +367,7 @@ __global__ void __cluster_dims__(4, 1, 1) __launch_bounds__(kLThreads, 1)
         // swap behind it: one-gate level 1.92 -> 1.83 ms)
         if (tid == kBkIssuer) {
             if (i + 2 < kn) {
-                mb_expect(&S.mbar_rows[buf], kRowsBytes);                     // rows / partial of step i + 2
+                mb_expect(&S.mbar_part[buf], kPartBytes);                     // partials of step i + 2
                 issue_bk_l(S, bkf, i + 2, o, q, h, buf);
             }
         }

@@ -20,14 +20,14 @@
 namespace tb {
 
 struct __align__(128) Brl2Smem {
-    double2 bk[2][kRows][512];                 // BK_i rows 0..5 of outputs o = 2q + h, h = 0, 1 (96 KB)
+    double2 bk[2][kRows][512];                 // BK_i (issue_bk_l2), h = 0, 1 (96 KB)
     double2 dslot[kL][512];                    // own forward rows (bloc q), swizzled positions
     double2 precv[2][2][512];                  // the partner's partial MACs of this CTA's outputs, by step parity
     double2 oslot[2][512];                     // MAC outputs (h = 0, 1), then the inverses' exchange buffers
     uint32_t res[2][kN];                       // rounded halves, h = 0 (lo) and 1 (hi, << 16)
     uint32_t acc[3 * kN];                      // ACC[q] as (acc, -acc, acc)
     uint16_t bar[kn + 2];
-    unsigned long long mbar_bk, mbar_rows[2];
+    unsigned long long mbar_bk, mbar_part[2];
 };
 
 // BK_i -> bk (one thread): slot (h, r) = the own bloc's row 3q + (r mod 3) of output 2q + h (r < 3) and of the
@@ -61,9 +61,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
 
     if (tid == 0) {
         mb_init(&S.mbar_bk);
-        for (int b = 0; b < 2; b++) mb_init(&S.mbar_rows[b]);
+        for (int b = 0; b < 2; b++) mb_init(&S.mbar_part[b]);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        for (int b = 0; b < 2; b++) mb_expect(&S.mbar_rows[b], 2 * 512 * 16);   // partials of steps 0 and 1
+        for (int b = 0; b < 2; b++) mb_expect(&S.mbar_part[b], 2 * 512 * 16);   // partials of steps 0 and 1
     }
     __syncthreads();
     if (tid == 0) issue_bk_l2(S, bkf, 0, q);
@@ -105,8 +105,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
     t3.a = ldc(twL + tt * 6 + 3);
     t3.b = ldc(twL + tt * 6 + 4);
     t3.c = ldc(twL + tt * 6 + 5);
-    const uint32_t rows_dst = cl_map(sm32(&S.precv[0][0][0]), rank ^ 1u);
-    const uint32_t rows_mb = cl_map(sm32(&S.mbar_rows[0]), rank ^ 1u);
+    const uint32_t part_dst = cl_map(sm32(&S.precv[0][0][0]), rank ^ 1u);
+    const uint32_t part_mb = cl_map(sm32(&S.mbar_part[0]), rank ^ 1u);
 
     for (int i = 0; i < kn; i++) {
         const int buf = i & 1;
@@ -144,12 +144,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
                     p1.im = fma(d.re, c1.im, fma(d.im, c1.re, p1.im));
                 }
                 asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f64 [%0], {%1, %2}, [%3];" ::"r"(
-                                 rows_dst + (uint32_t)(((buf * 2 + 0) * 512 + k) * 16)),
-                             "d"(p0.re), "d"(p0.im), "r"(rows_mb + (uint32_t)(buf * 8))
+                                 part_dst + (uint32_t)(((buf * 2 + 0) * 512 + k) * 16)),
+                             "d"(p0.re), "d"(p0.im), "r"(part_mb + (uint32_t)(buf * 8))
                              : "memory");
                 asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f64 [%0], {%1, %2}, [%3];" ::"r"(
-                                 rows_dst + (uint32_t)(((buf * 2 + 1) * 512 + k) * 16)),
-                             "d"(p1.re), "d"(p1.im), "r"(rows_mb + (uint32_t)(buf * 8))
+                                 part_dst + (uint32_t)(((buf * 2 + 1) * 512 + k) * 16)),
+                             "d"(p1.re), "d"(p1.im), "r"(part_mb + (uint32_t)(buf * 8))
                              : "memory");
 #pragma unroll
                 for (int r = 0; r < kL; r++) {
@@ -164,7 +164,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
             m3[e][0] = s0;
             m3[e][1] = s1;
         }
-        mb_wait(&S.mbar_rows[buf], par);
+        mb_wait(&S.mbar_part[buf], par);
 #pragma unroll
         for (int e = 0; e < kLMacIt; e++) {
             const int k = tid + kLThreads * e;
@@ -176,7 +176,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kLThreads, 1)
         }
         __syncthreads();                                  // bk, precv[buf] consumed; oslot complete
         if (tid == kBk2Issuer) {   // a thread of warp 4, idle during the two inverses (warp pairs 0 and 1)
-            if (i + 2 < kn) mb_expect(&S.mbar_rows[buf], 2 * 512 * 16);    // partials of step i + 2
+            if (i + 2 < kn) mb_expect(&S.mbar_part[buf], 2 * 512 * 16);    // partials of step i + 2
             if (i + 1 < kn) issue_bk_l2(S, bkf, i + 1, q);                  // lands during C and the next A
         }
         if (jd < 2) {   // ---- C: inverse of half h = jd (warp pair jd), round, << 16 h ----
